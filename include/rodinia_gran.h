@@ -1,0 +1,244 @@
+/*
+ * rodinia_gran.h -- C ABI of librodinia_gran.so: granularity-parameterised Rodinia kernels
+ * (hotspot, srad_v2, pathfinder, lud) for NVIDIA B200 (sm_100a).
+ *
+ * Source of the operations.  Ivanov et al., "Retargeting and Respecializing GPU Workloads
+ * for Performance Portability", CGO'24.  The paper takes
+ * existing CUDA kernels (Rodinia v3) and varies their *granularity*: the
+ * amount of work per thread (thread coarsening, §V-A) and the amount of
+ * work and shared memory per block (block coarsening, §V-B), emitting
+ * several alternatives (§VI), pruning them with ptxas register/spill data
+ * and choosing one by timing (TDO).  Coarsening never changes
+ * what a kernel computes.  Each entry point below therefore takes the
+ * plain Rodinia operation plus an explicit rodinia_granularity; DESIGN.md §3 lists every
+ * reading of the operations where the paper is silent.
+ *
+ * Conventions (all entry points):
+ *  - Buffers are DEVICE pointers (cudaMalloc / torch CUDA tensors), row-major, C-contiguous,
+ *    pitch = cols, owned and freed by the caller, unless the name ends in `_host`, in which
+ *    case they are plain host pointers and the call copies in/out itself (synchronous).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Device calls
+ *    are stream-ordered: they enqueue work and return; only `_host` calls, rodinia_tune and
+ *    rodinia_sync block.
+ *  - Errors are returned as rodinia_status, never thrown/aborted.  Argument errors are
+ *    detected before any CUDA call (so they are reported on hosts without a GPU too).
+ *    Asynchronous kernel faults surface at the next call or at rodinia_sync.
+ *    rodinia_last_error() returns a thread-local message for the last non-OK status.
+ *  - The library owns only internal scratch (ping-pong / coefficient buffers), allocated
+ *    stream-ordered (cudaMallocAsync) and freed stream-ordered before the call returns.
+ *  - Sizes are int64_t; rows, cols >= 1.  int32 overflow of pathfinder costs is the
+ *    caller's contract (as in Rodinia).
+ */
+#ifndef RODINIA_GRAN_H
+#define RODINIA_GRAN_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RODINIA_ABI_VERSION 1
+
+typedef enum {
+    RODINIA_OK = 0,
+    RODINIA_E_INVALID = -1,        /* null pointer, size < 1, iterations < 0, ROI outside grid,
+                                      lambda not finite, aliasing in/out buffers            */
+    RODINIA_E_ILLEGAL_FACTOR = -2, /* factor < 1; in FAITHFUL mode a thread factor that does not
+                                      divide the original tile; temporal depth
+                                      larger than the variant/slab supports                   */
+    RODINIA_E_SMEM = -3,           /* variant needs more shared memory per CTA than the device
+                                      offers (early pruning)                    */
+    RODINIA_E_FILTERED = -4,       /* variant rejected by the compile-time ptxas filter: new
+                                      spills or < 1 CTA/SM                     */
+    RODINIA_E_NOT_BUILT = -5,      /* factor combination not instantiated in this build       */
+    RODINIA_E_DEGENERATE = -6,     /* srad: ROI mean == 0, q0sqr undefined                     */
+    RODINIA_E_NODEV = -7,          /* no CUDA device / driver                                  */
+    RODINIA_E_CUDA = -8,           /* CUDA runtime error (message in rodinia_last_error)       */
+    RODINIA_E_NCCL = -9,           /* NCCL error or NCCL library not loadable                  */
+    RODINIA_E_NOMEM = -10          /* device or host allocation failed                         */
+} rodinia_status;
+
+/* Granularity of one kernel launch (§V).
+ *  thread_x/thread_y : thread-coarsening factor -- work units per thread along x / y
+ *                      (1 = uncoarsened).  CTA threads = original threads / (tx*ty), number of
+ *                      CTAs unchanged.
+ *  block_x/block_y   : block-coarsening factor -- original tiles merged into one CTA along
+ *                      x / y.  Threads per CTA unchanged, CTAs / (bx*by), shared memory x b
+ *                      (PAPER.md:185, 233).  Any value >= 1: remainder tiles are masked in
+ *                      the last CTA row/column (the paper's epilogue kernel).
+ *  temporal          : time steps fused per launch (hotspot / pathfinder pyramid height,
+ *                      srad fused depth); 1 = one step per launch.
+ *  index_mode        : 0 = coalescing-friendly (a thread's units are strided by the thread
+ *                      count, Fig.11 of the paper), 1 = contiguous (a thread's units are
+ *                      adjacent; 4 contiguous fp32 = one 128-bit access).
+ *  flags             : bit0 RODINIA_FAITHFUL -- paper factor rules only (thread factors must
+ *                      divide the original tile).
+ *                      bit1 RODINIA_STREAM -- use the streaming temporal-blocking family
+ *                      (hotspot).
+ * A NULL rodinia_granularity* (or all fields zero) selects the tuned variant from the tune
+ * cache if one exists for this (device, kernel, shape), else the built-in default. */
+typedef struct {
+    int32_t thread_x, thread_y;
+    int32_t block_x, block_y;
+    int32_t temporal;
+    int32_t index_mode;
+    int32_t flags;
+} rodinia_granularity;
+
+#define RODINIA_FAITHFUL 1
+#define RODINIA_STREAM 2
+
+typedef enum { RODINIA_HOTSPOT = 0, RODINIA_SRAD = 1, RODINIA_PATHFINDER = 2, RODINIA_LUD = 3 } rodinia_kernel;
+
+/* ---------------------------------------------------------------------------------------
+ * hotspot -- Rodinia hotspot `calculate_temp` (2-D thermal RC stencil), see DESIGN.md §3 H1-H8.
+ * One step, every cell (clamped neighbours, Jacobi):
+ *   T'[i][j] = c + k*( P[i][j] + ((S+N) - 2c)*ry + ((E+W) - 2c)*rx + (amb - c)*rz ),
+ *   c = T[i][j], N/S/W/E = T[i-+1][j], T[i][j-+1] clamped to the grid.
+ * `k, rx, ry, rz, amb` are explicit (reading H1: Rodinia's fixed 16 mm chip makes the step
+ * unstable above ~1386^2 cells).  k = step/Cap, r* = 1/R*.
+ */
+typedef struct { float k, rx, ry, rz, amb; } rodinia_hotspot_coeffs;
+
+/* Rodinia's chip formulas (H1) in fp64 for a chip_w x chip_h metre die, each
+ * coefficient rounded to fp32 once.  Pure host arithmetic. */
+rodinia_status rodinia_hotspot_coeffs_rodinia(int64_t rows, int64_t cols, double chip_w_m,
+                                              double chip_h_m, rodinia_hotspot_coeffs* out);
+
+/* `iterations` steps from temp_in (never written) into temp_out (must not alias temp_in).
+ * power: rows x cols.  scratch: NULL or a rows*cols fp32 device buffer used as the
+ * ping-pong partner (else allocated stream-ordered).  coeffs NULL => Rodinia 16 mm chip.
+ * iterations == 0 copies temp_in to temp_out. */
+rodinia_status rodinia_hotspot(const float* temp_in, const float* power, float* temp_out,
+                               float* scratch, int64_t rows, int64_t cols, int32_t iterations,
+                               const rodinia_hotspot_coeffs* coeffs,
+                               const rodinia_granularity* g, void* stream);
+
+/* Same with HOST buffers: H2D copy of temp_in and power, the solve, D2H copy of the result,
+ * all inside the call (synchronous).  Device buffers are cached inside the library. */
+rodinia_status rodinia_hotspot_host(const float* temp_in, const float* power, float* temp_out,
+                                    int64_t rows, int64_t cols, int32_t iterations,
+                                    const rodinia_hotspot_coeffs* coeffs,
+                                    const rodinia_granularity* g, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * srad_v2 -- Rodinia srad_v2 (speckle-reducing anisotropic diffusion), DESIGN.md §3 S1-S9.
+ * Per iteration: q0sqr = var/mean^2 of J over the ROI rows r1..r2, cols c1..c2 (inclusive),
+ * summed in fp64, rounded to fp32 once; pass 1 computes the clamped diffusion coefficient c
+ * of every cell from the old J; pass 2 updates J += 0.25*lambda*(c*dN + c_S*dS + c*dW +
+ * c_E*dE) (Jacobi).  J (rows x cols, values > 0) is updated in place.
+ * Returns RODINIA_E_DEGENERATE if the ROI mean becomes 0 (checked on the device; reported at
+ * the next call / rodinia_sync as the sticky status, J left as of the failing iteration).
+ */
+rodinia_status rodinia_srad(float* J, int64_t rows, int64_t cols, int64_t r1, int64_t r2,
+                            int64_t c1, int64_t c2, float lambda, int32_t niter,
+                            const rodinia_granularity* g, void* stream);
+rodinia_status rodinia_srad_host(float* J, int64_t rows, int64_t cols, int64_t r1, int64_t r2,
+                                 int64_t c1, int64_t c2, float lambda, int32_t niter,
+                                 const rodinia_granularity* g, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * pathfinder -- Rodinia pathfinder `dynproc_kernel` (min-cost path DP), P1-P6.
+ *   prev = wall[0]; next[j] = wall[r][j] + min(prev[j-1], prev[j], prev[j+1]) (existing
+ *   indices), r = 1..rows-1; result (cols int32) = prev after the last row.  Bit-exact. */
+rodinia_status rodinia_pathfinder(const int32_t* wall, int64_t rows, int64_t cols,
+                                  int32_t* result, const rodinia_granularity* g, void* stream);
+rodinia_status rodinia_pathfinder_host(const int32_t* wall, int64_t rows, int64_t cols,
+                                       int32_t* result, const rodinia_granularity* g,
+                                       void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * lud -- Rodinia lud (blocked Doolittle LU, no pivoting), L1-L6.  a (n x n fp32)
+ * is factored in place: unit-diagonal L strictly below the diagonal, U on and above.
+ * panel: block (panel) width; 16 = Rodinia's BLOCK_SIZE (0 => 16).  Supported: 16, 32.
+ * The panel width changes fp32 rounding order and is reported separately from coarsening
+ * (reading L5).  Zero pivots give inf/NaN (no pivoting, as Rodinia). */
+rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
+                           void* stream);
+rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel,
+                                const rodinia_granularity* g, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Variants, compile-time filter and timing-driven tuning (§VI, 251-269).
+ */
+typedef struct {
+    int64_t rows, cols;      /* lud: rows = cols = n; pathfinder: rows x cols wall */
+    int32_t iterations;      /* hotspot / srad iterations (tuning times min(iterations, 50)) */
+    int32_t nranks;          /* 1 for single-GPU problems; part of the cache key */
+} rodinia_problem;
+
+typedef struct {
+    rodinia_granularity g;
+    float median_ms;         /* tune rows only; -1 when not timed */
+    int32_t regs;            /* registers / thread (ptxas) */
+    int32_t spill_bytes;     /* spill stores + loads (ptxas) */
+    int32_t smem_bytes;      /* static + dynamic shared memory per CTA at this shape */
+    int32_t threads;         /* threads per CTA */
+    int32_t ctas_per_sm;     /* occupancy (runtime query; 0 when no device) */
+    int32_t status;          /* RODINIA_OK, or why the variant is pruned */
+} rodinia_tune_row;
+
+/* Enumerate the instantiated variants of kernel k with their ptxas statistics and the
+ * compile-time filter decision.  *n: in = capacity of out (may be 0), out = number of
+ * variants.  Pure host call (no device needed). */
+rodinia_status rodinia_variants(rodinia_kernel k, rodinia_tune_row* out, int32_t* n);
+
+/* Time every surviving variant on synthetic inputs of the problem's shape (never the
+ * caller's buffers): `reps` timed runs after one warm-up, CUDA events, median, argmin.
+ * Writes the winner to *best and stores it in the tune cache ($RODINIA_TUNE_CACHE, JSON
+ * lines, keyed by device name, SM count, kernel, shape, nranks).  rows/nrows as above. */
+rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* p, int32_t reps,
+                            rodinia_granularity* best, rodinia_tune_row* rows,
+                            int32_t* nrows);
+
+/* Resolve what a NULL/zero granularity would run for this problem (cache or default). */
+rodinia_status rodinia_resolve(rodinia_kernel k, const rodinia_problem* p,
+                               rodinia_granularity* out);
+
+/* ---------------------------------------------------------------------------------------
+ * Multi-GPU row-slab decomposition (hotspot, srad), one process per GPU.  The NCCL
+ * communicator is bootstrapped from a unique id the caller distributes (e.g. with
+ * torch.distributed.broadcast_object_list).  NCCL is loaded at run time (dlopen of the
+ * libnccl.so.2 already mapped by torch, else $RODINIA_NCCL_LIB).
+ * Rank r owns global rows [floor(r*R/P), floor((r+1)*R/P)).
+ */
+typedef struct rodinia_comm rodinia_comm;
+
+rodinia_status rodinia_slab(int64_t global_rows, int32_t nranks, int32_t rank, int64_t* row0,
+                            int64_t* nrows);
+rodinia_status rodinia_comm_unique_id(uint8_t id[128]);
+rodinia_status rodinia_comm_init(rodinia_comm** out, int32_t nranks, int32_t rank,
+                                 const uint8_t id[128]);
+/* In-process "loopback" communicator: `nranks` slabs on the current device, halos moved
+ * with cudaMemcpyAsync (tests the decomposition on one GPU). */
+rodinia_status rodinia_comm_init_local(rodinia_comm** out, int32_t nranks);
+rodinia_status rodinia_comm_destroy(rodinia_comm* comm);
+
+/* NCCL communicator: temp_local/power_local/out_local hold this rank's slab (rodinia_slab
+ * rows x cols).  Local communicator: the pointers are arrays of `nranks` slab pointers
+ * (const float* const*), passed as the same arguments.  Bitwise equal to rodinia_hotspot
+ * on the whole grid with the same granularity. */
+rodinia_status rodinia_hotspot_dist(rodinia_comm* comm, const void* temp_local,
+                                    const void* power_local, void* out_local,
+                                    int64_t global_rows, int64_t cols, int32_t iterations,
+                                    const rodinia_hotspot_coeffs* coeffs,
+                                    const rodinia_granularity* g, void* stream);
+rodinia_status rodinia_srad_dist(rodinia_comm* comm, void* J_local, int64_t global_rows,
+                                 int64_t cols, int64_t r1, int64_t r2, int64_t c1, int64_t c2,
+                                 float lambda, int32_t niter, const rodinia_granularity* g,
+                                 void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Misc. */
+const char* rodinia_last_error(void);
+const char* rodinia_status_string(rodinia_status s);
+rodinia_status rodinia_sync(void* stream);          /* stream sync + sticky async errors */
+int32_t rodinia_abi_version(void);
+/* Number of kernel launches this library has issued since load (for bench accounting). */
+int64_t rodinia_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RODINIA_GRAN_H */

@@ -1,0 +1,435 @@
+// hotspot.cu -- granularity-parameterised hotspot kernels for sm_100a.
+//
+// Operation: Rodinia hotspot `calculate_temp` (DESIGN.md §3 H1-H8), per cell via hs_cell().
+// Two variant families:
+//
+//  * hs_direct<TX,TY,MODE>  (temporal = 1).  The paper's granularity space verbatim: the
+//    original kernel is a 16x16-thread CTA computing one 16x16 tile, one cell per thread.
+//    Thread coarsening (TX,TY) gives each thread TX x TY cells of its tile and shrinks the CTA
+//    to (16/TX) x (16/TY) threads, #CTAs unchanged.  Block coarsening
+//    (bx,by, runtime) merges bx x by tiles into one CTA, threads unchanged, #CTAs / (bx*by)
+//    (PAPER.md:181-185); ragged edges are masked (the paper's epilogue).
+//    MODE 0 = coalescing-friendly indexing (a thread's cells are NTX apart), MODE 1 =
+//    contiguous cells (TX % 4 == 0 -> 128-bit loads/stores) (Fig. 11).
+//    Neighbours are read straight from global memory (L1 serves the reuse): at one step per
+//    launch the kernel is HBM-bound at 12 B per cell-update.
+//
+//  * hs_stream<V,H>  (temporal = H >= 2), the B200 temporal-blocking family.  Each warp owns a
+//    band of 32*V staged columns (V contiguous columns per lane, 128-bit accesses) and streams
+//    down a chunk of rows; H time levels are kept in registers as 3-row rings and advance one
+//    row per step with a lag of one row per level, so H steps of the stencil cost one HBM read
+//    of T and P and one write of T'.  E/W neighbours come from warp shuffles, N/S from the
+//    register rings; no shared memory and no block barriers.  The band overlaps its neighbours
+//    by H columns on each side (redundant halo compute), the chunk by H rows above and below.
+//    Results are bit-identical to H applications of hs_direct (same hs_cell, same operands).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+
+#include "hs_cell.cuh"
+#include "rg_internal.h"
+
+namespace rg {
+
+__device__ __forceinline__ float4 ldg4(const float* p) {
+    return __ldg(reinterpret_cast<const float4*>(p));
+}
+__device__ __forceinline__ void stg4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+
+// ============================================================================ direct family
+// ptxas otherwise budgets registers for 2048 resident threads (32 regs) and spills the
+// coarsened variants; ask for >= 1024 resident threads (<= 64 regs) instead.
+template <int TX, int TY, int MODE>
+__global__ void __launch_bounds__((16 / TX) * (16 / TY),
+                                  (1024 / ((16 / TX) * (16 / TY))) < 32 ? (1024 / ((16 / TX) * (16 / TY))) : 32)
+    hs_direct(const float* __restrict__ tin, const float* __restrict__ pw,
+              float* __restrict__ tout, int R, int C, int bx, int by, HsCoef cf, int vec_ok) {
+    constexpr int NTX = 16 / TX, NTY = 16 / TY;
+    const int x0 = blockIdx.x * 16 * bx;
+    const int y0 = blockIdx.y * 16 * by;
+    for (int b_y = 0; b_y < by; ++b_y) {
+#pragma unroll
+        for (int t_y = 0; t_y < TY; ++t_y) {
+            const int row = y0 + b_y * 16 +
+                            (MODE == 0 ? (int)threadIdx.y + t_y * NTY : (int)threadIdx.y * TY + t_y);
+            if (row >= R) continue;
+            const size_t rc = (size_t)row * C;
+            const size_t rn = (size_t)max(row - 1, 0) * C;
+            const size_t rs = (size_t)min(row + 1, R - 1) * C;
+            for (int b_x = 0; b_x < bx; ++b_x) {
+                const int xt = x0 + b_x * 16;
+                if (MODE == 1) {
+                    const int col0 = xt + (int)threadIdx.x * TX;
+                    if ((TX % 4 == 0) && vec_ok && col0 + TX <= C) {
+#pragma unroll
+                        for (int q = 0; q < TX / 4; ++q) {
+                            const int cq = col0 + 4 * q;
+                            const float4 c4 = ldg4(tin + rc + cq);
+                            const float4 n4 = ldg4(tin + rn + cq);
+                            const float4 s4 = ldg4(tin + rs + cq);
+                            const float4 p4 = ldg4(pw + rc + cq);
+                            const float w = cq > 0 ? __ldg(tin + rc + cq - 1) : c4.x;
+                            const float e = cq + 4 < C ? __ldg(tin + rc + cq + 4) : c4.w;
+                            float4 o;
+                            o.x = hs_cell(c4.x, n4.x, s4.x, c4.y, w, p4.x, cf);
+                            o.y = hs_cell(c4.y, n4.y, s4.y, c4.z, c4.x, p4.y, cf);
+                            o.z = hs_cell(c4.z, n4.z, s4.z, c4.w, c4.y, p4.z, cf);
+                            o.w = hs_cell(c4.w, n4.w, s4.w, e, c4.z, p4.w, cf);
+                            stg4(tout + rc + cq, o);
+                        }
+                        continue;
+                    }
+                }
+#pragma unroll
+                for (int t_x = 0; t_x < TX; ++t_x) {
+                    const int col = MODE == 0 ? xt + (int)threadIdx.x + t_x * NTX
+                                              : xt + (int)threadIdx.x * TX + t_x;
+                    if (col >= C) continue;
+                    const int cw = max(col - 1, 0), ce = min(col + 1, C - 1);
+                    const float c = __ldg(tin + rc + col);
+                    tout[rc + col] = hs_cell(c, __ldg(tin + rn + col), __ldg(tin + rs + col),
+                                             __ldg(tin + rc + ce), __ldg(tin + rc + cw),
+                                             __ldg(pw + rc + col), cf);
+                }
+            }
+        }
+    }
+}
+
+// ============================================================================ stream family
+// Per-lane register state: ring[l][slot][v] holds level l (0 = input T) at three consecutive
+// rows; at step s (level-0 row g0 = ystart + s) level l's newest row g0 - l sits in slot
+// (s+2)%3, row g0-l-1 in (s+1)%3 and row g0-l-2 in s%3.  The step loop is unrolled by 3 so
+// every ring index is a compile-time constant (no register moves).
+//
+// Fast path (EC = ER = false, the vast majority of warps): the band lies inside the grid with
+// aligned vector access and the chunk's staged rows lie strictly inside the grid, so there are
+// no bounds checks and no clamps; every branch below is warp-uniform.
+//   EC: band touches a grid column edge (or vector access impossible) -> scalar, column clamp.
+//   ER: chunk's staged rows reach row 0 or R-1 -> row checks and row clamp.
+template <int V>
+struct VecT;
+template <> struct VecT<1> { typedef float T; };
+template <> struct VecT<2> { typedef float2 T; };
+template <> struct VecT<4> { typedef float4 T; };
+
+template <int V, bool EC, bool ER>
+__device__ __forceinline__ void hs_ld(const float* __restrict__ base, int row, int R, int C, int col0,
+                                      float (&out)[V]) {
+    if (ER && (row < 0 || row >= R)) {
+#pragma unroll
+        for (int v = 0; v < V; ++v) out[v] = 0.0f;
+        return;
+    }
+    const float* p = base + (size_t)row * C + col0;
+    if (!EC) {
+        const typename VecT<V>::T t = __ldg(reinterpret_cast<const typename VecT<V>::T*>(p));
+        const float* f = reinterpret_cast<const float*>(&t);
+#pragma unroll
+        for (int v = 0; v < V; ++v) out[v] = f[v];
+    } else {
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            const int c = col0 + v;
+            out[v] = (c >= 0 && c < C) ? __ldg(p + v) : 0.0f;
+        }
+    }
+}
+
+template <int V, int H, int K, bool EC, bool ER>
+__device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&nxt_t)[V],
+                                               float (&nxt_p)[V], const float* __restrict__ tin,
+                                               const float* __restrict__ pw, float* __restrict__ tout,
+                                               int g0, int R, int C, int ylo, int yhi, int sc0, int col0,
+                                               const HsCoef& cf) {
+    constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
+    // level 0: the prefetched row g0 becomes the newest level-0 row; prefetch T row g0+1 and the
+    // power row g0 (needed by level 1 at the next step).
+    float p1[V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) { ring[0][S2][v] = nxt_t[v]; p1[v] = nxt_p[v]; }
+    hs_ld<V, EC, ER>(tin, g0 + 1, R, C, col0, nxt_t);
+    hs_ld<V, EC, ER>(pw, g0, R, C, col0, nxt_p);
+
+#pragma unroll
+    for (int l = 0; l < H; ++l) {
+        const int g = g0 - l - 1;  // row computed by level l+1
+        float pv[V];
+        if (l == 0) {
+#pragma unroll
+            for (int v = 0; v < V; ++v) pv[v] = p1[v];
+        } else {
+            hs_ld<V, EC, ER>(pw, g, R, C, col0, pv);  // L1 hit: first touched by level 1
+        }
+        const bool top = ER && (g == 0), bot = ER && (g == R - 1);
+        const float wnb = __shfl_up_sync(0xffffffffu, ring[l][S1][V - 1], 1);
+        const float enb = __shfl_down_sync(0xffffffffu, ring[l][S1][0], 1);
+        float res[V];
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            const float c = ring[l][S1][v];
+            const float n = top ? c : ring[l][S0][v];
+            const float s = bot ? c : ring[l][S2][v];
+            float w = v > 0 ? ring[l][S1][v > 0 ? v - 1 : 0] : wnb;
+            float e = v < V - 1 ? ring[l][S1][v < V - 1 ? v + 1 : 0] : enb;
+            if (EC) {
+                const int col = col0 + v;
+                if (col == 0) w = c;
+                if (col == C - 1) e = c;
+            }
+            res[v] = hs_cell(c, n, s, e, w, pv[v], cf);
+        }
+        if (l + 1 < H) {
+#pragma unroll
+            for (int v = 0; v < V; ++v) ring[l + 1 < H ? l + 1 : 0][S2][v] = res[v];
+        } else if (g >= ylo && g < yhi) {
+            // level H: write the lane's cells that lie in the band's output columns
+            constexpr int s_lo = H, s_hi = 32 * V - H;  // staged-column range of the output
+            float* orow = tout + (size_t)g * C + col0;
+            if (!EC && (H % V == 0)) {
+                if (sc0 >= s_lo && sc0 < s_hi) {
+                    typename VecT<V>::T t;
+                    float* f = reinterpret_cast<float*>(&t);
+#pragma unroll
+                    for (int v = 0; v < V; ++v) f[v] = res[v];
+                    *reinterpret_cast<typename VecT<V>::T*>(orow) = t;
+                }
+            } else {
+#pragma unroll
+                for (int v = 0; v < V; ++v) {
+                    const int col = col0 + v;
+                    if (sc0 + v >= s_lo && sc0 + v < s_hi && col >= 0 && col < C) orow[v] = res[v];
+                }
+            }
+        }
+    }
+}
+
+template <int V, int H, bool EC, bool ER>
+__device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
+                                               const float* __restrict__ pw,
+                                               float* __restrict__ tout, int R, int C, int y0,
+                                               int y1, int sc0, int col0, const HsCoef& cf) {
+    float ring[H][3][V];
+#pragma unroll
+    for (int l = 0; l < H; ++l)
+#pragma unroll
+        for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int v = 0; v < V; ++v) ring[l][k][v] = 0.0f;
+    const int ystart = y0 - H;
+    const int nsteps = (y1 - y0) + 2 * H;
+    float nxt_t[V], nxt_p[V];
+    hs_ld<V, EC, ER>(tin, ystart, R, C, col0, nxt_t);
+    hs_ld<V, EC, ER>(pw, ystart - 1, R, C, col0, nxt_p);
+    int s = 0;
+    for (; s + 3 <= nsteps; s += 3) {
+        hs_stream_step<V, H, 0, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 1, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 2, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 2, R, C, y0, y1, sc0, col0, cf);
+    }
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s, R, C, y0, y1, sc0, col0, cf);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
+}
+
+// One warp per CTA: every branch condition derives from blockIdx and kernel arguments only, so
+// the compiler sees it as warp-uniform and the shuffles need no convergence handling.  Block
+// coarsening along x (bands_per_cta) makes the warp process several adjacent bands in turn;
+// block coarsening along y is the chunk height (rows streamed per CTA).
+template <int V, int H>
+__global__ void __launch_bounds__(32, (V * H >= 32) ? 8 : 16)
+    hs_stream(const float* __restrict__ tin, const float* __restrict__ pw,
+              float* __restrict__ tout, int R, int C, int chunk, int bands_per_cta, HsCoef cf,
+              int vec_ok) {
+    constexpr int SW = 32 * V;
+    constexpr int OW = SW - 2 * H;
+    static_assert(OW > 0, "band narrower than its halo");
+    const int sc0 = (int)threadIdx.x * V;
+    const int y0 = blockIdx.y * chunk;
+    const int y1 = min(y0 + chunk, R);
+    const bool er = (y0 - H - 1 < 0) || (y1 + H > R - 1);
+    for (int bi = 0; bi < bands_per_cta; ++bi) {
+        const int band = blockIdx.x * bands_per_cta + bi;
+        if (band * OW >= C) return;
+        const int bstart = band * OW - H;
+        const int col0 = bstart + sc0;
+        const bool ec = !vec_ok || bstart < 0 || bstart + SW > C;
+        if (!ec && !er)
+            hs_stream_body<V, H, false, false>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+        else if (ec && !er)
+            hs_stream_body<V, H, true, false>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+        else if (!ec && er)
+            hs_stream_body<V, H, false, true>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+        else
+            hs_stream_body<V, H, true, true>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+    }
+}
+
+// ============================================================================ registry
+namespace hotspot {
+
+typedef void (*DirectFn)(const float*, const float*, float*, int, int, int, int, HsCoef, int);
+typedef void (*StreamFn)(const float*, const float*, float*, int, int, int, int, HsCoef, int);
+
+struct DirectVariant { int tx, ty, mode; DirectFn fn; const char* key; };
+struct StreamVariant { int v, h; StreamFn fn; const char* key; };
+
+#define RG_HSD(TX, TY, M) {TX, TY, M, hs_direct<TX, TY, M>, "void rg::hs_direct<" #TX ", " #TY ", " #M ">"}
+#define RG_HSD2(TX, TY) RG_HSD(TX, TY, 0), RG_HSD(TX, TY, 1)
+static const DirectVariant kDirect[] = {
+    RG_HSD2(1, 1),  RG_HSD2(1, 2), RG_HSD2(1, 4), RG_HSD2(1, 8), RG_HSD2(1, 16),
+    RG_HSD2(2, 1),  RG_HSD2(2, 2), RG_HSD2(2, 4), RG_HSD2(2, 8), RG_HSD2(2, 16),
+    RG_HSD2(4, 1),  RG_HSD2(4, 2), RG_HSD2(4, 4), RG_HSD2(4, 8),
+    RG_HSD2(8, 1),  RG_HSD2(8, 2), RG_HSD2(8, 4),
+    RG_HSD2(16, 1), RG_HSD2(16, 2),
+};
+#undef RG_HSD2
+#undef RG_HSD
+
+#define RG_HSS(V, H) {V, H, hs_stream<V, H>, "void rg::hs_stream<" #V ", " #H ">"}
+static const StreamVariant kStream[] = {
+    RG_HSS(4, 2), RG_HSS(4, 4), RG_HSS(4, 6), RG_HSS(4, 8), RG_HSS(4, 12), RG_HSS(4, 16),
+    RG_HSS(2, 4), RG_HSS(2, 8),
+    RG_HSS(1, 4), RG_HSS(1, 8),
+};
+#undef RG_HSS
+
+const DirectVariant* find_direct(int tx, int ty, int mode) {
+    for (const auto& v : kDirect)
+        if (v.tx == tx && v.ty == ty && v.mode == mode) return &v;
+    return nullptr;
+}
+const StreamVariant* find_stream(int v_, int h) {
+    for (const auto& v : kStream)
+        if (v.v == v_ && v.h == h) return &v;
+    return nullptr;
+}
+
+static bool is_div16(int t) { return t == 1 || t == 2 || t == 4 || t == 8 || t == 16; }
+
+// Host-only legality check (no CUDA call).  Fills the variant pointers.
+rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C,
+                     const DirectVariant** dv, const StreamVariant** sv) {
+    *dv = nullptr; *sv = nullptr;
+    if (g.thread_x < 1 || g.thread_y < 1 || g.block_x < 1 || g.block_y < 1 || g.temporal < 1)
+        return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: factors must be >= 1 (%s)", gran_str(g).c_str());
+    if (g.index_mode != 0 && g.index_mode != 1)
+        return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: index_mode must be 0 or 1");
+    const bool stream = (g.flags & RODINIA_STREAM) != 0;
+    if (!stream) {
+        if (g.temporal != 1)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR,
+                             "hotspot: the direct family fuses one step per launch (temporal=1); "
+                             "set RODINIA_STREAM for temporal blocking");
+        if (!is_div16(g.thread_x) || !is_div16(g.thread_y))
+            return set_error(RODINIA_E_ILLEGAL_FACTOR,
+                             "hotspot: thread factors must divide the 16x16 tile (PAPER.md:237)");
+        if (g.block_x > 4096 || g.block_y > 4096)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: block factor too large");
+        const int64_t gy = ((R + 15) / 16 + g.block_y - 1) / g.block_y;
+        if (gy > 65535)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: grid.y %lld > 65535; raise block_y", (long long)gy);
+        *dv = find_direct(g.thread_x, g.thread_y, g.index_mode);
+        if (!*dv)
+            return set_error(RODINIA_E_NOT_BUILT, "hotspot: direct variant %s not instantiated", gran_str(g).c_str());
+    } else {
+        if (g.flags & RODINIA_FAITHFUL)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: the stream family is not a faithful-mode variant");
+        if (g.thread_y != 1 || g.index_mode != 1)
+            return set_error(RODINIA_E_NOT_BUILT, "hotspot: stream family needs thread_y=1, index_mode=1");
+        if (g.temporal < 2)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: stream family needs temporal >= 2");
+        if (g.block_x > 4096)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: stream block_x too large");
+        const int64_t chunk = 16 * (int64_t)g.block_y;
+        if ((R + chunk - 1) / chunk > 65535)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: too many row chunks; raise block_y");
+        *sv = find_stream(g.thread_x, g.temporal);
+        if (!*sv)
+            return set_error(RODINIA_E_NOT_BUILT, "hotspot: stream variant %s not instantiated", gran_str(g).c_str());
+    }
+    return RODINIA_OK;
+}
+
+static void launch_direct(const DirectVariant* dv, int bx, int by, const float* tin, const float* p,
+                          float* tout, int R, int C, const HsCoef& cf, cudaStream_t s) {
+    const int tiles_x = (C + 15) / 16, tiles_y = (R + 15) / 16;
+    dim3 grid((tiles_x + bx - 1) / bx, (tiles_y + by - 1) / by);
+    dim3 block(16 / dv->tx, 16 / dv->ty);
+    const int vec_ok = (C % 4 == 0) &&
+                       ((reinterpret_cast<uintptr_t>(tin) | reinterpret_cast<uintptr_t>(p) |
+                         reinterpret_cast<uintptr_t>(tout)) % 16 == 0);
+    dv->fn<<<grid, block, 0, s>>>(tin, p, tout, R, C, bx, by, cf, vec_ok);
+    count_launch();
+}
+
+static void launch_stream(const StreamVariant* sv, int bx, int by, const float* tin, const float* p,
+                          float* tout, int R, int C, const HsCoef& cf, cudaStream_t s) {
+    const int ow = 32 * sv->v - 2 * sv->h;
+    const int bands = (C + ow - 1) / ow;
+    const int chunk = 16 * by;
+    dim3 grid((bands + bx - 1) / bx, (R + chunk - 1) / chunk);
+    // vector access needs every lane's first column aligned to V floats
+    const int vec_ok = (C % sv->v == 0) && (sv->h % sv->v == 0) &&
+                       ((reinterpret_cast<uintptr_t>(tin) | reinterpret_cast<uintptr_t>(p) |
+                         reinterpret_cast<uintptr_t>(tout)) % (4 * sv->v) == 0);
+    sv->fn<<<grid, 32, 0, s>>>(tin, p, tout, R, C, chunk, bx, cf, vec_ok);
+    count_launch();
+}
+
+// Run `iters` steps on a (R x C) buffer from `tin` into `tout`, ping-ponging through `scr`.
+// The granularity has been validated by check().  Neighbour rows are clamped to the buffer,
+// so the same routine serves whole grids and halo'd slabs.
+rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C,
+                   int iters, const HsCoef& cf, const rodinia_granularity& g,
+                   const DirectVariant* dv, const StreamVariant* sv, cudaStream_t s) {
+    if (iters == 0) {
+        RG_CUDA(cudaMemcpyAsync(tout, tin, (size_t)R * C * sizeof(float), cudaMemcpyDeviceToDevice, s));
+        return RODINIA_OK;
+    }
+    const int h = sv ? sv->h : 1;
+    const int nfull = iters / h, rem = iters % h;
+    const int launches = nfull + rem;  // remainder steps run one per launch (direct family)
+    const DirectVariant* remv = find_direct(4, 1, 1);
+    int left = launches;
+    const float* src = tin;
+    int done = 0;
+    while (left > 0) {
+        float* dst = ((left - 1) % 2 == 0) ? tout : scr;
+        if (sv && done < nfull) {
+            launch_stream(sv, g.block_x, g.block_y, src, p, dst, R, C, cf, s);
+            ++done;
+        } else if (dv) {
+            launch_direct(dv, g.block_x, g.block_y, src, p, dst, R, C, cf, s);
+        } else {
+            launch_direct(remv, 1, 1, src, p, dst, R, C, cf, s);
+        }
+        src = dst;
+        --left;
+    }
+    RG_CUDA(cudaGetLastError());
+    return RODINIA_OK;
+}
+
+int num_variants() { return (int)(sizeof(kDirect) / sizeof(kDirect[0]) + sizeof(kStream) / sizeof(kStream[0])); }
+
+// Describe variant i: granularity (block factors 1), kernel pointer, key, threads per CTA.
+void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    const int nd = (int)(sizeof(kDirect) / sizeof(kDirect[0]));
+    if (i < nd) {
+        const auto& v = kDirect[i];
+        *g = gran(v.tx, v.ty, 1, 1, 1, v.mode);
+        *fn = (const void*)v.fn;
+        *key = v.key;
+        *threads = (16 / v.tx) * (16 / v.ty);
+    } else {
+        const auto& v = kStream[i - nd];
+        *g = gran(v.v, 1, 1, 16, v.h, 1, RODINIA_STREAM);
+        *fn = (const void*)v.fn;
+        *key = v.key;
+        *threads = 32;
+    }
+}
+
+}  // namespace hotspot
+}  // namespace rg

@@ -1,0 +1,296 @@
+// tune.cu -- variant enumeration with the compile-time (ptxas) filter, and the timing-driven
+// tuner (TDO): every surviving alternative is run on synthetic data of the
+// problem's shape, timed with CUDA events (one warm-up, `reps` timed runs, median), the
+// fastest is returned and cached.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "hs_cell.cuh"
+#include "rg_internal.h"
+
+namespace rg {
+
+extern const PtxasStats kPtxasStats[];
+extern const int kNumPtxasStats;
+
+const PtxasStats* find_stats(const char* key) {
+    for (int i = 0; i < kNumPtxasStats; ++i)
+        if (strcmp(kPtxasStats[i].key, key) == 0) return &kPtxasStats[i];
+    return nullptr;
+}
+
+// ---------------------------------------------------------------- per-workload registries
+namespace hotspot {
+struct DirectVariant;
+struct StreamVariant;
+int num_variants();
+void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads);
+rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C, const DirectVariant** dv,
+                     const StreamVariant** sv);
+rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C, int iters,
+                   const HsCoef& cf, const rodinia_granularity& g, const DirectVariant* dv,
+                   const StreamVariant* sv, cudaStream_t s);
+}  // namespace hotspot
+
+struct Registry {
+    int (*count)();
+    void (*info)(int, rodinia_granularity*, const void**, const char**, int*);
+};
+
+// Filled in by the other workload TUs through these hooks.
+int srad_num_variants();
+void srad_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
+int pathfinder_num_variants();
+void pathfinder_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
+int lud_num_variants();
+void lud_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
+
+static Registry registry(rodinia_kernel k) {
+    switch (k) {
+        case RODINIA_HOTSPOT: return {hotspot::num_variants, hotspot::variant_info};
+        case RODINIA_SRAD: return {srad_num_variants, srad_variant_info};
+        case RODINIA_PATHFINDER: return {pathfinder_num_variants, pathfinder_variant_info};
+        case RODINIA_LUD: return {lud_num_variants, lud_variant_info};
+    }
+    return {nullptr, nullptr};
+}
+
+static void fill_row(rodinia_kernel k, int i, bool have_dev, int base_spill, rodinia_tune_row* r) {
+    Registry reg = registry(k);
+    const void* fn;
+    const char* key;
+    int threads;
+    memset(r, 0, sizeof *r);
+    reg.info(i, &r->g, &fn, &key, &threads);
+    const PtxasStats* st = find_stats(key);
+    r->median_ms = -1.0f;
+    r->regs = st ? st->regs : -1;
+    r->spill_bytes = st ? st->spill_stores + st->spill_loads : -1;
+    r->smem_bytes = st ? st->smem : -1;
+    r->threads = threads;
+    r->ctas_per_sm = have_dev ? ctas_per_sm(fn, threads, 0) : 0;
+    r->status = filter_decision(st, threads, 0, base_spill);
+    if (r->status == RODINIA_OK && have_dev && r->ctas_per_sm == 0) r->status = RODINIA_E_FILTERED;
+}
+
+static int family_base_spill(rodinia_kernel k) {
+    // The uncoarsened kernel of each workload is variant 0 of its registry.
+    Registry reg = registry(k);
+    if (reg.count() == 0) return 0;
+    rodinia_granularity g;
+    const void* fn;
+    const char* key;
+    int threads;
+    reg.info(0, &g, &fn, &key, &threads);
+    const PtxasStats* st = find_stats(key);
+    return st ? st->spill_stores + st->spill_loads : 0;
+}
+
+rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
+    switch (k) {
+        case RODINIA_HOTSPOT:
+            // B200 default: streaming temporal blocking, 4 columns per lane,
+            // 8 steps per launch, 4 warps per CTA, 256-row chunks.
+            if (p.iterations >= 8 && p.cols >= 128) return gran(4, 1, 4, 16, 8, 1, RODINIA_STREAM);
+            return gran(4, 1, 1, 1, 1, 1);
+        case RODINIA_SRAD: return gran(4, 1, 1, 1, 1, 1);
+        case RODINIA_PATHFINDER: return gran(4, 1, 1, 1, 8, 1);
+        case RODINIA_LUD: return gran(1, 1, 1, 1, 1, 0);
+    }
+    return gran(1, 1, 1, 1, 1, 0);
+}
+
+// ---------------------------------------------------------------- synthetic data
+__global__ void rg_fill(float* a, int64_t n, float base, float scale, uint32_t seed) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t x = (uint32_t)i * 2654435761u ^ seed;
+        x ^= x >> 13; x *= 0x5bd1e995u; x ^= x >> 15;
+        a[i] = base + scale * (float)(x & 0xffffff) * (1.0f / 16777216.0f);
+    }
+}
+
+static rodinia_status fill(float* a, int64_t n, float base, float scale, uint32_t seed, cudaStream_t s) {
+    rg_fill<<<1184, 256, 0, s>>>(a, n, base, scale, seed);
+    RG_CUDA(cudaGetLastError());
+    return RODINIA_OK;
+}
+
+// Candidate granularities to time for hotspot (each combined with the instantiated variants).
+static void hotspot_candidates(const rodinia_problem& p, std::vector<rodinia_granularity>* out) {
+    const int n = hotspot::num_variants();
+    for (int i = 0; i < n; ++i) {
+        rodinia_granularity g;
+        const void* fn;
+        const char* key;
+        int threads;
+        hotspot::variant_info(i, &g, &fn, &key, &threads);
+        if (g.flags & RODINIA_STREAM) {
+            for (int w : {2, 4, 8})
+                for (int by : {8, 16, 32}) {
+                    g.block_x = w;
+                    g.block_y = by;
+                    out->push_back(g);
+                }
+        } else {
+            static const int bxy[][2] = {{1, 1}, {2, 1}, {4, 1}, {1, 2}, {2, 2}, {7, 1}, {8, 1}, {4, 4}};
+            for (auto& b : bxy) {
+                g.block_x = b[0];
+                g.block_y = b[1];
+                out->push_back(g);
+            }
+        }
+    }
+    (void)p;
+}
+
+static float median(std::vector<float> v) {
+    std::sort(v.begin(), v.end());
+    return v.empty() ? -1.f : v[v.size() / 2];
+}
+
+static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_granularity* best,
+                                   std::vector<rodinia_tune_row>* rows) {
+    const int64_t R = p.rows, C = p.cols;
+    const int iters = std::max(1, std::min(p.iterations, 48));
+    cudaStream_t s;
+    RG_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    float *tin = nullptr, *pw = nullptr, *tout = nullptr, *scr = nullptr;
+    const size_t bytes = (size_t)R * C * sizeof(float);
+    rodinia_status st = RODINIA_OK;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    if (cudaMalloc(&tin, bytes) != cudaSuccess || cudaMalloc(&pw, bytes) != cudaSuccess ||
+        cudaMalloc(&tout, bytes) != cudaSuccess || cudaMalloc(&scr, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        st = set_error(RODINIA_E_NOMEM, "tune: cannot allocate %zu-byte buffers", bytes);
+    }
+    if (st == RODINIA_OK) st = fill(tin, R * C, 323.15f, 20.0f, 1u, s);
+    if (st == RODINIA_OK) st = fill(pw, R * C, 0.0f, 1e-3f, 2u, s);
+    rodinia_hotspot_coeffs cc;
+    rodinia_hotspot_coeffs_rodinia(R, C, R * 31.25e-6, C * 31.25e-6, &cc);
+    const HsCoef cf{cc.k, cc.rx, cc.ry, cc.rz, cc.amb};
+    std::vector<rodinia_granularity> cands;
+    hotspot_candidates(p, &cands);
+    const int base_spill = family_base_spill(RODINIA_HOTSPOT);
+    float best_ms = 1e30f;
+    for (size_t ci = 0; st == RODINIA_OK && ci < cands.size(); ++ci) {
+        rodinia_tune_row row;
+        memset(&row, 0, sizeof row);
+        row.g = cands[ci];
+        row.median_ms = -1.f;
+        const hotspot::DirectVariant* dv;
+        const hotspot::StreamVariant* sv;
+        rodinia_status cs = hotspot::check(row.g, R, C, &dv, &sv);
+        if (cs == RODINIA_OK) {
+            // ptxas statistics / filter of the underlying instantiation
+            const int n = hotspot::num_variants();
+            for (int i = 0; i < n; ++i) {
+                rodinia_granularity g;
+                const void* fn;
+                const char* key;
+                int threads;
+                hotspot::variant_info(i, &g, &fn, &key, &threads);
+                if (g.thread_x == row.g.thread_x && g.thread_y == row.g.thread_y &&
+                    g.temporal == row.g.temporal && g.index_mode == row.g.index_mode &&
+                    (g.flags & RODINIA_STREAM) == (row.g.flags & RODINIA_STREAM)) {
+                    const PtxasStats* ps = find_stats(key);
+                    if (g.flags & RODINIA_STREAM) threads = 32 * row.g.block_x;
+                    row.regs = ps ? ps->regs : -1;
+                    row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
+                    row.smem_bytes = ps ? ps->smem : -1;
+                    row.threads = threads;
+                    row.ctas_per_sm = ctas_per_sm(fn, threads, 0);
+                    cs = filter_decision(ps, threads, 0, base_spill);
+                    if (cs == RODINIA_OK && row.ctas_per_sm == 0) cs = RODINIA_E_FILTERED;
+                    break;
+                }
+            }
+        }
+        if (cs == RODINIA_OK) {
+            std::vector<float> ts;
+            for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {
+                cudaEventRecord(e0, s);
+                cs = hotspot::run(tin, pw, tout, scr, (int)R, (int)C, iters, cf, row.g, dv, sv, s);
+                cudaEventRecord(e1, s);
+                if (cudaEventSynchronize(e1) != cudaSuccess) {
+                    cs = cuda_error(cudaGetLastError(), "tune run", __FILE__, __LINE__);
+                    st = cs;  // a faulting variant is a hard error
+                }
+                float ms = 0;
+                cudaEventElapsedTime(&ms, e0, e1);
+                if (r >= 0) ts.push_back(ms);
+            }
+            if (cs == RODINIA_OK) {
+                row.median_ms = median(ts);
+                if (row.median_ms < best_ms) { best_ms = row.median_ms; *best = row.g; }
+            }
+        }
+        row.status = cs;
+        rows->push_back(row);
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(tin); cudaFree(pw); cudaFree(tout); cudaFree(scr);
+    cudaStreamDestroy(s);
+    if (st == RODINIA_OK && best_ms >= 1e29f) st = set_error(RODINIA_E_FILTERED, "tune: no variant survived");
+    if (st == RODINIA_OK) tune_cache_store(RODINIA_HOTSPOT, p, *best, best_ms);
+    return st;
+}
+
+rodinia_status tune_srad(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
+rodinia_status tune_pathfinder(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
+rodinia_status tune_lud(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
+
+}  // namespace rg
+
+using namespace rg;
+
+extern "C" rodinia_status rodinia_variants(rodinia_kernel k, rodinia_tune_row* out, int32_t* n) {
+    if (!n || *n < 0 || (*n > 0 && !out)) return set_error(RODINIA_E_INVALID, "variants: bad arguments");
+    if ((int)k < 0 || (int)k > 3) return set_error(RODINIA_E_INVALID, "variants: unknown kernel %d", (int)k);
+    Registry reg = registry(k);
+    const int total = reg.count();
+    int cnt = 0;
+    cudaGetDeviceCount(&cnt);
+    cudaGetLastError();
+    const bool have_dev = cnt > 0;
+    const int base_spill = family_base_spill(k);
+    for (int i = 0; i < total && i < *n; ++i) fill_row(k, i, have_dev, base_spill, &out[i]);
+    *n = total;
+    return RODINIA_OK;
+}
+
+extern "C" rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* p, int32_t reps,
+                                       rodinia_granularity* best, rodinia_tune_row* rows, int32_t* nrows) {
+    if (!p || !best || reps < 1 || p->rows < 1 || p->cols < 1 || p->iterations < 0 || p->nranks < 1)
+        return set_error(RODINIA_E_INVALID, "tune: bad arguments");
+    if (nrows && *nrows > 0 && !rows) return set_error(RODINIA_E_INVALID, "tune: rows is null");
+    if ((int)k < 0 || (int)k > 3) return set_error(RODINIA_E_INVALID, "tune: unknown kernel %d", (int)k);
+    DeviceInfo di;
+    RG_TRY(device_info(&di));
+    std::vector<rodinia_tune_row> out;
+    rodinia_status st;
+    switch (k) {
+        case RODINIA_HOTSPOT: st = tune_hotspot(*p, reps, best, &out); break;
+        case RODINIA_SRAD: st = tune_srad(*p, reps, best, &out); break;
+        case RODINIA_PATHFINDER: st = tune_pathfinder(*p, reps, best, &out); break;
+        default: st = tune_lud(*p, reps, best, &out); break;
+    }
+    if (nrows) {
+        const int cap = *nrows;
+        for (int i = 0; i < cap && i < (int)out.size(); ++i) rows[i] = out[i];
+        *nrows = (int)out.size();
+    }
+    return st;
+}
+
+extern "C" rodinia_status rodinia_resolve(rodinia_kernel k, const rodinia_problem* p, rodinia_granularity* out) {
+    if (!p || !out) return set_error(RODINIA_E_INVALID, "resolve: bad arguments");
+    if (tune_cache_lookup(k, *p, out)) return RODINIA_OK;
+    *out = default_gran(k, *p);
+    return RODINIA_OK;
+}
