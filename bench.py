@@ -1,0 +1,451 @@
+#!/usr/bin/env python
+"""bench.py -- headline benchmark: hotspot 16384x16384 fp32, 1000 iterations (BASELINE.json
+configs[2]), cell-updates/s, through the C ABI of librodinia_gran.so.
+
+One "step" = one full hotspot solve (1000 Jacobi iterations of the whole grid) with the
+timing-driven (autotuned) granularity; inputs resident in HBM before the timed
+region.  `e2e` repeats the solve through rodinia_hotspot_host() with pinned host buffers
+(H2D of T and P, the solve, D2H of T' inside the timed region).  The uncoarsened
+one-cell-per-thread variant and the other workloads (srad, pathfinder, lud) are measured in
+the same run and reported under "workloads", with the geomean speedup tuned/uncoarsened.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--no-tune] [--no-extra] [--rows R] [--iters I]
+
+Multi-GPU (torchrun, one rank per GPU): row slabs with NCCL halo exchange
+(rodinia_hotspot_dist); timing = max over ranks of CUDA-event time around the K steps.
+`--impl reference` times the CPU oracle (the plain C definition, oracle/) on a bounded sample
+of the same workload on this host's cores -- the only reference this paper-only tier has.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "hotspot/srad cell-updates/s at 1–8 GPUs; geomean speedup vs uncoarsened"
+UNC = (1, 1, 1, 1, 1, 0, 0)
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return d.get("hbm_gbs", 6650.0), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """Samples nvidia-smi clocks and throttle reasons during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- dist helpers
+def _dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _max_over_ranks(x: float, ws: int) -> float:
+    if ws == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def _barrier(ws):
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+# ----------------------------------------------------------------------------- CPU reference
+def cpu_oracle_hotspot(rows_sample: int, cols: int, iters: int, N: int):
+    """Time the fp64 C oracle on a bounded sample (rows_sample x cols, `iters` steps)."""
+    import numpy as np
+
+    import oracle
+    import synth
+    T, P = synth.hotspot_inputs(rows_sample, cols)
+    c = oracle.hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6)
+    T64, P64 = T.astype(np.float64), P.astype(np.float64)
+    t0 = time.perf_counter()
+    oracle.hotspot(T64, P64, iters, **c)
+    dt = time.perf_counter() - t0
+    return rows_sample * cols * iters / dt, dt
+
+
+def run_reference(args):
+    ws, rank, _ = _dist_env()
+    if rank != 0:
+        return 0
+    N, iters_full = args.rows, args.iters
+    rows_sample = 1024
+    rate0, dt0 = cpu_oracle_hotspot(rows_sample, N, 1, N)  # calibration
+    it = max(1, min(50, int(round(6.0 / max(dt0, 1e-3)))))  # ~6 s per step
+    for _ in range(args.warmup):
+        cpu_oracle_hotspot(rows_sample, N, max(1, it // 4), N)
+    rates, times = [], []
+    for _ in range(args.steps):
+        r, dt = cpu_oracle_hotspot(rows_sample, N, it, N)
+        rates.append(r)
+        times.append(dt)
+    v = statistics.median(rates)
+    sample = f"{rows_sample}x{N} rows x cols, {it} iterations per step (of the {N}x{N}x{iters_full} workload), fp64 plain C"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "cell-updates/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": statistics.median(times) * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"hotspot {N}x{N} fp32, {iters_full} iterations (CPU oracle sample)",
+                   "rows": N, "cols": N, "iterations": iters_full},
+        "cpu_baseline": {"value": v, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": v, "unit": "cell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------- GPU arm
+def _time_steps(fn, steps, warmup, stream):
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / steps
+
+
+def extra_workloads(rg, torch, tune: bool):
+    """srad / pathfinder / lud at their BASELINE configs (1 GPU): tuned vs uncoarsened."""
+    out = {}
+    s = torch.cuda.current_stream()
+    have = {n: hasattr(rg, "rodinia_" + n) for n in ("srad", "pathfinder", "lud")}
+
+    def timed(fn, reps=5):
+        fn()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(reps):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            fn()
+            e1.record(s)
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        return statistics.median(ts)
+
+    # srad_v2 8192^2, 100 iterations, ROI (0,127,0,127), lambda 0.5
+    try:
+        import synth
+        n, it = 8192, 100
+        J0 = torch.from_numpy(synth.srad_input(n, n)).cuda()
+        J = J0.clone()
+        res = {}
+        for name, g in (("uncoarsened", UNC), ("tuned", None)):
+            if name == "tuned" and tune:
+                g, _ = rg.rodinia_tune("srad", n, n, it, reps=2)
+            ms = timed(lambda: (J.copy_(J0), rg.rodinia_srad(J, 0, 127, 0, 127, 0.5, it, g=g)))
+            res[name] = {"ms": ms, "cell_updates_per_s": n * n * it / (ms * 1e-3),
+                         "g": list(g.astuple()) if hasattr(g, "astuple") else (list(g) if g else None)}
+        res["speedup"] = res["uncoarsened"]["ms"] / res["tuned"]["ms"]
+        out["srad"] = res
+    except Exception as e:  # noqa: BLE001
+        out["srad"] = {"error": str(e)[:200]}
+    # pathfinder 100 rows x 100000 cols int32, per-call time over batches
+    try:
+        import synth
+        w = torch.from_numpy(synth.pathfinder_wall(100, 100000)).cuda()
+        r = torch.empty(100000, dtype=torch.int32, device="cuda")
+        res = {}
+        for name, g in (("uncoarsened", (1, 1, 1, 1, 20, 0, 0)), ("tuned", None)):
+            if name == "tuned" and tune:
+                g, _ = rg.rodinia_tune("pathfinder", 100, 100000, 1, reps=3)
+            # one call is ~10 us of GPU work: time a CUDA graph of `batch` calls so host-side
+            # launch overhead does not pollute the per-call device time (PAPER.md:305 drops
+            # runs under 1e-4 s for the same reason)
+            batch = 200
+            rg.rodinia_pathfinder(w, g=g, out=r)
+            gs = torch.cuda.Stream()
+            gs.wait_stream(s)
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.stream(gs):
+                with torch.cuda.graph(graph, stream=gs):
+                    for _ in range(batch):
+                        rg.rodinia_pathfinder(w, g=g, out=r)
+            torch.cuda.synchronize()
+            ms = timed(graph.replay) / batch
+            res[name] = {"ms_per_call": ms, "cell_updates_per_s": 99 * 100000 / (ms * 1e-3),
+                         "g": list(g.astuple()) if hasattr(g, "astuple") else list(g)}
+        res["speedup"] = res["uncoarsened"]["ms_per_call"] / res["tuned"]["ms_per_call"]
+        out["pathfinder"] = res
+    except Exception as e:  # noqa: BLE001
+        out["pathfinder"] = {"error": str(e)[:200]}
+    # lud 8192^2 fp32
+    try:
+        import synth
+        n = 8192
+        A0 = torch.from_numpy(synth.lud_rodinia_matrix(n)).cuda()
+        A = A0.clone()
+        res = {}
+        for name, g in (("uncoarsened", UNC), ("tuned", None)):
+            if name == "tuned" and tune:
+                g, _ = rg.rodinia_tune("lud", n, n, 1, reps=2)
+            ms = timed(lambda: (A.copy_(A0), rg.rodinia_lud(A, 16, g=g)), reps=3)
+            res[name] = {"ms": ms, "gflops": (2 * n ** 3 / 3) / (ms * 1e-3) / 1e9,
+                         "g": list(g.astuple()) if hasattr(g, "astuple") else list(g)}
+        res["speedup"] = res["uncoarsened"]["ms"] / res["tuned"]["ms"]
+        out["lud"] = res
+    except Exception as e:  # noqa: BLE001
+        out["lud"] = {"error": str(e)[:200]}
+    return out
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+
+    ws, rank, local = _dist_env()
+    torch.cuda.set_device(local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_cgo_ivanovzdem24_b200 as rg
+    import synth
+
+    N, iters = args.rows, args.iters
+    stream = torch.cuda.current_stream()
+    coef = rg.rodinia_hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6)  # reading H1
+
+    # ---- tuning (TDO) on synthetic data of the problem's shape, before the timed region
+    t_tune = time.perf_counter()
+    if args.no_tune:
+        g = rg.rodinia_resolve("hotspot", N, N, iters, ws)
+        tune_rows = []
+    else:
+        g, tune_rows = rg.rodinia_tune("hotspot", N if ws == 1 else N // ws, N, iters, nranks=1, reps=2)
+    t_tune = time.perf_counter() - t_tune
+
+    T, P = synth.hotspot_inputs(N, N)
+    if ws == 1:
+        t = torch.from_numpy(T).cuda()
+        p = torch.from_numpy(P).cuda()
+        out = torch.empty_like(t)
+        scr = torch.empty_like(t)
+        def step(gg=g):
+            rg.rodinia_hotspot(t, p, iters, coeffs=coef, g=gg, out=out, scratch=scr, stream=stream)
+    else:
+        comm = rg.dist.HaloComm.from_process_group()
+        r0, nr = rg.rodinia_slab(N, ws, rank)
+        t = torch.from_numpy(T[r0:r0 + nr]).cuda()
+        p = torch.from_numpy(P[r0:r0 + nr]).cuda()
+        out = torch.empty_like(t)
+        def step(gg=g):
+            comm.hotspot(t, p, out, N, iters, coeffs=coef, g=gg, stream=stream)
+    del T, P
+
+    # ---- timed region (device events, max over ranks)
+    _barrier(ws)
+    torch.cuda.synchronize()
+    l0 = rg.rodinia_launch_count()
+    with ClockSampler(local) as clk:
+        ms = _time_steps(step, args.steps, args.warmup, stream)
+    launches_total = rg.rodinia_launch_count() - l0
+    launches_timed = launches_total * args.steps // (args.steps + args.warmup)
+    ms = _max_over_ranks(ms, ws)
+    _barrier(ws)
+    value = N * N * iters / (ms * 1e-3)
+
+    # ---- roofline of the dominant kernel (one kernel type per step, no remainder launches
+    # when iters % temporal == 0): avg launch duration = step time / launches per step.
+    h = g.temporal if g.temporal >= 1 else 1
+    launches_per_step = launches_timed / args.steps
+    rows_local = N if ws == 1 else N // ws
+    hbm_peak, peak_src = _peaks()
+    bytes_per_launch = 12.0 * rows_local * N  # algorithmic: read T, read P, write T'
+    avg_launch_ms = ms / max(launches_per_step, 1)
+    achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "r01_hotspot_traffic.json")
+    if os.path.exists(tp):
+        try:
+            with open(tp) as f:
+                traffic = json.load(f).get("traffic_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+            "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
+            "kernel": "hs_stream" if g.flags & rg.RODINIA_STREAM else "hs_direct",
+            "bytes_per_launch": bytes_per_launch, "avg_launch_ms": avg_launch_ms,
+            "updates_per_launch": rows_local * N * h}
+
+    # ---- uncoarsened variant (same timed protocol, fewer steps)
+    unc_ms = None
+    if not args.no_extra:
+        unc_ms = _max_over_ranks(_time_steps(lambda: step(UNC), 1, 1, stream), ws)
+
+    result = None
+    if rank == 0:
+        # ---- e2e through the C ABI with pinned host buffers (1 GPU)
+        e2e = None
+        if ws == 1:
+            th = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+            ph = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+            oh = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+            th.copy_(t.cpu()); ph.copy_(p.cpu())
+            thn, phn, ohn = th.numpy(), ph.numpy(), oh.numpy()
+            rg.rodinia_hotspot_host(thn, phn, iters, coeffs=coef, g=g, out=ohn)
+            e2e_t = []
+            for _ in range(max(1, min(args.steps, 3))):
+                t0 = time.perf_counter()
+                rg.rodinia_hotspot_host(thn, phn, iters, coeffs=coef, g=g, out=ohn)
+                e2e_t.append(time.perf_counter() - t0)
+            e2e_s = statistics.median(e2e_t)
+            e2e = {"value": N * N * iters / e2e_s, "unit": "cell-updates/s",
+                   "h2d_bytes_per_step": 2 * 4 * N * N, "d2h_bytes_per_step": 4 * N * N,
+                   "ms_per_step": e2e_s * 1e3}
+            assert np.isfinite(ohn[::997, ::991]).all()
+        # ---- CPU oracle baseline (bounded sample)
+        cpu = None
+        if not args.no_cpu:
+            r1, d1 = cpu_oracle_hotspot(1024, N, 1, N)
+            it = max(1, min(40, int(round(12.0 / max(d1, 1e-3)))))
+            rate, dt = cpu_oracle_hotspot(1024, N, it, N)
+            cpu = {"value": rate, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
+                   "sample": f"1024x{N} rows x cols of the {N}x{N} grid, {it} iterations "
+                             f"({dt:.1f} s), fp64 plain C, single thread"}
+        extra = extra_workloads(rg, torch, not args.no_tune) if (ws == 1 and not args.no_extra) else {}
+        speedups = {"hotspot": (unc_ms / ms) if unc_ms else None}
+        for k, v in extra.items():
+            if isinstance(v, dict) and "speedup" in v:
+                speedups[k] = v["speedup"]
+        sp = [x for x in speedups.values() if x]
+        geomean = float(np.exp(np.mean(np.log(sp)))) if sp else None
+        clocks = clk.summary()
+        result = {
+            "metric": METRIC, "value": value, "unit": "cell-updates/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": f"hotspot {N}x{N} fp32, {iters} iterations (BASELINE configs[2])",
+                       "rows": N, "cols": N, "iterations": iters,
+                       "coefficients": "512-grid cell size (DESIGN.md H1)",
+                       "granularity": list(g.astuple()),
+                       "parallelism": f"row-slab x{ws}" if ws > 1 else "single GPU",
+                       "l2": "no flush: working set 3 GiB >> 126 MB L2",
+                       "tune_seconds": round(t_tune, 1)},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches_timed,
+            "clocks": clocks,
+            "uncoarsened": {"ms_per_step": unc_ms,
+                            "value": N * N * iters / (unc_ms * 1e-3) if unc_ms else None},
+            "speedup_vs_uncoarsened": speedups,
+            "geomean_speedup_vs_uncoarsened": geomean,
+            "workloads": extra,
+            "paper_context": "27% Rodinia geomean speedup, A100/A4000, composite timing (PAPER.md:29)",
+        }
+        print(json.dumps(result), flush=True)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--rows", type=int, default=16384)
+    ap.add_argument("--iters", type=int, default=1000)
+    ap.add_argument("--no-tune", action="store_true")
+    ap.add_argument("--no-extra", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -76,6 +76,11 @@ typedef enum {
  *                      divide the original tile).
  *                      bit1 RODINIA_STREAM -- use the streaming temporal-blocking family
  *                      (hotspot).
+ *                      bits 8..15 RODINIA_OCC(n) -- register budget of the instantiation:
+ *                      target n resident CTAs per SM (launch bounds => <= 65536/(threads*n)
+ *                      registers per thread); 0 = the family's preferred instantiation.  This
+ *                      is the register/occupancy trade-off the paper can only observe through
+ *                      ptxas; here it is an explicit alternative.
  * A NULL rodinia_granularity* (or all fields zero) selects the tuned variant from the tune
  * cache if one exists for this (device, kernel, shape), else the built-in default. */
 typedef struct {
@@ -88,6 +93,8 @@ typedef struct {
 
 #define RODINIA_FAITHFUL 1
 #define RODINIA_STREAM 2
+#define RODINIA_OCC(n) (((n) & 0xff) << 8)
+#define RODINIA_OCC_OF(flags) (((flags) >> 8) & 0xff)
 
 typedef enum { RODINIA_HOTSPOT = 0, RODINIA_SRAD = 1, RODINIA_PATHFINDER = 2, RODINIA_LUD = 3 } rodinia_kernel;
 

@@ -237,12 +237,14 @@ extern "C" const char* rodinia_status_string(rodinia_status s) {
 extern "C" int32_t rodinia_abi_version(void) { return RODINIA_ABI_VERSION; }
 extern "C" int64_t rodinia_launch_count(void) { return g_launches.load(); }
 
+namespace rg { namespace srad { rodinia_status take_sticky(); } }
+
 extern "C" rodinia_status rodinia_sync(void* stream) {
     DeviceInfo di;
     RG_TRY(device_info(&di));
     RG_CUDA(cudaStreamSynchronize((cudaStream_t)stream));
     RG_CUDA(cudaGetLastError());
-    return RODINIA_OK;
+    return srad::take_sticky();
 }
 
 // ===================================================================== exported: hotspot

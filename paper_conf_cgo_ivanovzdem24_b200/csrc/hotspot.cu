@@ -236,8 +236,8 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
 // the compiler sees it as warp-uniform and the shuffles need no convergence handling.  Block
 // coarsening along x (bands_per_cta) makes the warp process several adjacent bands in turn;
 // block coarsening along y is the chunk height (rows streamed per CTA).
-template <int V, int H>
-__global__ void __launch_bounds__(32, (V * H >= 32) ? 8 : 16)
+template <int V, int H, int OCC>
+__global__ void __launch_bounds__(32, OCC)
     hs_stream(const float* __restrict__ tin, const float* __restrict__ pw,
               float* __restrict__ tout, int R, int C, int chunk, int bands_per_cta, HsCoef cf,
               int vec_ok) {
@@ -272,7 +272,7 @@ typedef void (*DirectFn)(const float*, const float*, float*, int, int, int, int,
 typedef void (*StreamFn)(const float*, const float*, float*, int, int, int, int, HsCoef, int);
 
 struct DirectVariant { int tx, ty, mode; DirectFn fn; const char* key; };
-struct StreamVariant { int v, h; StreamFn fn; const char* key; };
+struct StreamVariant { int v, h, occ; StreamFn fn; const char* key; };
 
 #define RG_HSD(TX, TY, M) {TX, TY, M, hs_direct<TX, TY, M>, "void rg::hs_direct<" #TX ", " #TY ", " #M ">"}
 #define RG_HSD2(TX, TY) RG_HSD(TX, TY, 0), RG_HSD(TX, TY, 1)
@@ -286,11 +286,17 @@ static const DirectVariant kDirect[] = {
 #undef RG_HSD2
 #undef RG_HSD
 
-#define RG_HSS(V, H) {V, H, hs_stream<V, H>, "void rg::hs_stream<" #V ", " #H ">"}
+#define RG_HSS(V, H, O) {V, H, O, hs_stream<V, H, O>, "void rg::hs_stream<" #V ", " #H ", " #O ">"}
 static const StreamVariant kStream[] = {
-    RG_HSS(4, 2), RG_HSS(4, 4), RG_HSS(4, 6), RG_HSS(4, 8), RG_HSS(4, 12), RG_HSS(4, 16),
-    RG_HSS(2, 4), RG_HSS(2, 8),
-    RG_HSS(1, 4), RG_HSS(1, 8),
+    RG_HSS(4, 2, 16), RG_HSS(4, 2, 24),
+    RG_HSS(4, 4, 12), RG_HSS(4, 4, 16), RG_HSS(4, 4, 20), RG_HSS(4, 4, 24),
+    RG_HSS(4, 6, 10), RG_HSS(4, 6, 12), RG_HSS(4, 6, 16),
+    RG_HSS(4, 8, 8), RG_HSS(4, 8, 10), RG_HSS(4, 8, 12), RG_HSS(4, 8, 16),
+    RG_HSS(2, 4, 16), RG_HSS(2, 4, 24), RG_HSS(2, 4, 32),
+    RG_HSS(2, 8, 12), RG_HSS(2, 8, 16), RG_HSS(2, 8, 20), RG_HSS(2, 8, 24),
+    RG_HSS(2, 12, 12), RG_HSS(2, 12, 16),
+    RG_HSS(2, 16, 8), RG_HSS(2, 16, 12),
+    RG_HSS(1, 4, 16), RG_HSS(1, 8, 16),
 };
 #undef RG_HSS
 
@@ -299,9 +305,10 @@ const DirectVariant* find_direct(int tx, int ty, int mode) {
         if (v.tx == tx && v.ty == ty && v.mode == mode) return &v;
     return nullptr;
 }
-const StreamVariant* find_stream(int v_, int h) {
+// occ == 0 selects the first instantiation of (V, H) in kStream (ordered by preference).
+const StreamVariant* find_stream(int v_, int h, int occ) {
     for (const auto& v : kStream)
-        if (v.v == v_ && v.h == h) return &v;
+        if (v.v == v_ && v.h == h && (occ == 0 || v.occ == occ)) return &v;
     return nullptr;
 }
 
@@ -344,7 +351,7 @@ rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C,
         const int64_t chunk = 16 * (int64_t)g.block_y;
         if ((R + chunk - 1) / chunk > 65535)
             return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot: too many row chunks; raise block_y");
-        *sv = find_stream(g.thread_x, g.temporal);
+        *sv = find_stream(g.thread_x, g.temporal, RODINIA_OCC_OF(g.flags));
         if (!*sv)
             return set_error(RODINIA_E_NOT_BUILT, "hotspot: stream variant %s not instantiated", gran_str(g).c_str());
     }
@@ -424,7 +431,7 @@ void variant_info(int i, rodinia_granularity* g, const void** fn, const char** k
         *threads = (16 / v.tx) * (16 / v.ty);
     } else {
         const auto& v = kStream[i - nd];
-        *g = gran(v.v, 1, 1, 16, v.h, 1, RODINIA_STREAM);
+        *g = gran(v.v, 1, 1, 4, v.h, 1, RODINIA_STREAM | RODINIA_OCC(v.occ));
         *fn = (const void*)v.fn;
         *key = v.key;
         *threads = 32;

@@ -1,0 +1,420 @@
+// lud.cu -- granularity-parameterised blocked LU (Rodinia lud) for sm_100a.
+//
+// Operation: Doolittle LU without pivoting, packed in place (DESIGN.md §3 L1-L6), computed
+// with Rodinia's blocked structure.  For panel step k (offset o = P*k):
+//   lud_diag      in-tile Doolittle of the P x P diagonal tile (one CTA);
+//   lud_perim     U12 = L11^-1 A12 (unit-lower forward substitution) for every tile right of
+//                 the diagonal, L21 = A21 U11^-1 for every tile below it;
+//   lud_internal  A22 -= L21 * U12 for every trailing tile (the paper's "main lud kernel",
+//                 PAPER.md:315-353, which its coarsening study targets).
+// Granularity (§V) applies to lud_internal: thread coarsening (TX,TY) gives each thread
+// TX x TY elements of a tile and shrinks the CTA to (P/TX) x (P/TY) threads; block coarsening
+// (bx,by) merges bx x by trailing tiles into one CTA, whose shared memory holds bx U12 tiles
+// and by L21 tiles (shared memory x b).  The uncoarsened variant is Rodinia's:
+// P = 16, 16 x 16 threads, one element per thread, one tile per CTA.  The per-element
+// accumulation order (sum over i ascending, then a -= sum) is the same in every variant, so
+// for a fixed panel width every (t, b) variant is bit-identical (reading L5).
+//
+// The 3*ceil(n/P)-2 launches of one factorisation are captured once into a CUDA graph per
+// (device, n, P, granularity) and replayed; kernels read the matrix pointer from a device slot
+// the call sets first, so one graph serves every matrix of that size.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <map>
+#include <mutex>
+#include <tuple>
+#include <vector>
+
+#include "rg_internal.h"
+
+namespace rg {
+
+// ------------------------------------------------------------------ diagonal tile
+template <int P>
+__global__ void __launch_bounds__(P) lud_diag(float* const* __restrict__ slot, int n, int k) {
+    float* A = *slot;
+    __shared__ float t[P][P + 1];
+    const int o = k * P, r = min(P, n - o), tx = threadIdx.x;
+    for (int i = 0; i < r; ++i)
+        if (tx < r) t[i][tx] = A[(size_t)(o + i) * n + o + tx];
+    __syncthreads();
+    for (int i = 0; i < r - 1; ++i) {
+        if (tx > i && tx < r) {  // column i of L
+            float v = t[tx][i];
+            for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(t[tx][j], t[j][i]));
+            t[tx][i] = __fdiv_rn(v, t[i][i]);
+        }
+        __syncthreads();
+        if (tx > i && tx < r) {  // row i+1 of U
+            float v = t[i + 1][tx];
+            for (int j = 0; j < i + 1; ++j) v = __fsub_rn(v, __fmul_rn(t[i + 1][j], t[j][tx]));
+            t[i + 1][tx] = v;
+        }
+        __syncthreads();
+    }
+    for (int i = 0; i < r; ++i)
+        if (tx < r) A[(size_t)(o + i) * n + o + tx] = t[i][tx];
+}
+
+// ------------------------------------------------------------------ perimeter tiles
+// CTA j handles the j-th tile right of the diagonal (threads 0..P-1, one column each) and the
+// j-th tile below it (threads P..2P-1, one row each).
+template <int P>
+__global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
+    float* A = *slot;
+    __shared__ float dia[P][P + 1], row[P][P + 1], col[P][P + 1];
+    const int o = k * P;
+    const int r = P;  // diagonal tile is full whenever perimeter tiles exist
+    const int tb = o + P * (blockIdx.x + 1);  // first row/col of this perimeter tile
+    const int w = min(P, n - tb);             // its width (last tile may be partial)
+    const int tx = threadIdx.x;
+    if (tx < P) {
+        for (int i = 0; i < r; ++i) dia[i][tx] = A[(size_t)(o + i) * n + o + tx];
+        for (int i = 0; i < r; ++i) row[i][tx] = tx < w ? A[(size_t)(o + i) * n + tb + tx] : 0.f;
+    } else {
+        const int c = tx - P;
+        for (int i = 0; i < w; ++i) col[i][c] = A[(size_t)(tb + i) * n + o + c];
+    }
+    __syncthreads();
+    if (tx < P) {
+        if (tx < w)  // U12 column tx: forward substitution with unit-lower L11
+            for (int i = 1; i < r; ++i) {
+                float v = row[i][tx];
+                for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(dia[i][j], row[j][tx]));
+                row[i][tx] = v;
+            }
+    } else {
+        const int idx = tx - P;
+        if (idx < w)  // L21 row idx: solve against U11
+            for (int i = 0; i < r; ++i) {
+                float v = col[idx][i];
+                for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(col[idx][j], dia[j][i]));
+                col[idx][i] = __fdiv_rn(v, dia[i][i]);
+            }
+    }
+    __syncthreads();
+    if (tx < P) {
+        if (tx < w)
+            for (int i = 0; i < r; ++i) A[(size_t)(o + i) * n + tb + tx] = row[i][tx];
+    } else {
+        const int c = tx - P;
+        for (int i = 0; i < w; ++i) A[(size_t)(tb + i) * n + o + c] = col[i][c];
+    }
+}
+
+// ------------------------------------------------------------------ trailing update
+template <int P, int TX, int TY, int MODE>
+__global__ void __launch_bounds__((P / TX) * (P / TY),
+                                  (1024 / ((P / TX) * (P / TY))) < 32 ? (1024 / ((P / TX) * (P / TY))) : 32)
+    lud_internal(float* const* __restrict__ slot, int n, int k, int bx, int by) {
+    float* A = *slot;
+    extern __shared__ float lsm[];
+    constexpr int NTX = P / TX, NTY = P / TY, NT = NTX * NTY;
+    const int o = k * P;
+    const int t0 = o + P;  // first trailing row/col
+    const int cx0 = t0 + blockIdx.x * bx * P, cy0 = t0 + blockIdx.y * by * P;
+    float* Ush = lsm;                      // bx tiles of U12: [bx][P][P+1] (rows i, cols)
+    float* Lsh = lsm + bx * P * (P + 1);   // by tiles of L21: [by][P][P+1] (rows, i)
+    const int tid = threadIdx.y * NTX + threadIdx.x;
+    for (int e = tid; e < bx * P * P; e += NT) {
+        const int b = e / (P * P), rem = e - b * P * P, i = rem / P, c = rem - i * P;
+        const int gc = cx0 + b * P + c;
+        Ush[(b * P + i) * (P + 1) + c] = gc < n ? A[(size_t)(o + i) * n + gc] : 0.f;
+    }
+    for (int e = tid; e < by * P * P; e += NT) {
+        const int b = e / (P * P), rem = e - b * P * P, rr = rem / P, i = rem - rr * P;
+        const int gr = cy0 + b * P + rr;
+        Lsh[(b * P + rr) * (P + 1) + i] = gr < n ? A[(size_t)gr * n + o + i] : 0.f;
+    }
+    __syncthreads();
+    for (int b_y = 0; b_y < by; ++b_y)
+        for (int b_x = 0; b_x < bx; ++b_x)
+#pragma unroll
+            for (int t_y = 0; t_y < TY; ++t_y) {
+                const int ly = MODE == 0 ? (int)threadIdx.y + t_y * NTY : (int)threadIdx.y * TY + t_y;
+                const int gr = cy0 + b_y * P + ly;
+                float sum[TX];
+#pragma unroll
+                for (int t_x = 0; t_x < TX; ++t_x) sum[t_x] = 0.f;
+#pragma unroll 4
+                for (int i = 0; i < P; ++i) {
+                    const float l = Lsh[(b_y * P + ly) * (P + 1) + i];
+#pragma unroll
+                    for (int t_x = 0; t_x < TX; ++t_x) {
+                        const int lx = MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x;
+                        sum[t_x] = __fmaf_rn(l, Ush[(b_x * P + i) * (P + 1) + lx], sum[t_x]);
+                    }
+                }
+                if (gr < n) {
+#pragma unroll
+                    for (int t_x = 0; t_x < TX; ++t_x) {
+                        const int lx = MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x;
+                        const int gc = cx0 + b_x * P + lx;
+                        if (gc < n) {
+                            float* a = A + (size_t)gr * n + gc;
+                            *a = __fsub_rn(*a, sum[t_x]);
+                        }
+                    }
+                }
+            }
+}
+
+__global__ void lud_set_slot(float** slot, float* a) { *slot = a; }
+
+namespace lud {
+
+typedef void (*IntFn)(float* const*, int, int, int, int);
+typedef void (*DPFn)(float* const*, int, int);
+struct Variant { int p, tx, ty, mode; IntFn fn; const char* key; };
+
+#define RG_LI(P, TX, TY, M) {P, TX, TY, M, lud_internal<P, TX, TY, M>, "void rg::lud_internal<" #P ", " #TX ", " #TY ", " #M ">"}
+#define RG_LI2(P, TX, TY) RG_LI(P, TX, TY, 0), RG_LI(P, TX, TY, 1)
+static const Variant kInternal[] = {
+    RG_LI2(16, 1, 1), RG_LI2(16, 2, 1), RG_LI2(16, 1, 2), RG_LI2(16, 2, 2), RG_LI2(16, 4, 1),
+    RG_LI2(16, 1, 4), RG_LI2(16, 4, 2), RG_LI2(16, 2, 4), RG_LI2(16, 4, 4), RG_LI2(16, 8, 1),
+    RG_LI2(16, 8, 2), RG_LI2(16, 16, 1), RG_LI2(16, 16, 2),
+    RG_LI2(32, 1, 1), RG_LI2(32, 2, 1), RG_LI2(32, 2, 2), RG_LI2(32, 4, 1), RG_LI2(32, 4, 2),
+    RG_LI2(32, 4, 4), RG_LI2(32, 8, 2),
+};
+#undef RG_LI2
+#undef RG_LI
+
+static const Variant* find(int p, int tx, int ty, int mode) {
+    for (const auto& v : kInternal)
+        if (v.p == p && v.tx == tx && v.ty == ty && v.mode == mode) return &v;
+    return nullptr;
+}
+
+struct Plan {
+    int p;
+    const Variant* v;
+    int bx, by;
+    size_t smem;
+};
+
+rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
+    if (panel == 0) panel = 16;
+    if (panel != 16 && panel != 32)
+        return set_error(RODINIA_E_NOT_BUILT, "lud: panel width %d not built (16, 32)", panel);
+    if (g.thread_x < 1 || g.thread_y < 1 || g.block_x < 1 || g.block_y < 1 || g.temporal != 1)
+        return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: factors must be >= 1, temporal = 1 (%s)", gran_str(g).c_str());
+    if (g.index_mode != 0 && g.index_mode != 1)
+        return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: index_mode must be 0 or 1");
+    if (panel % g.thread_x || panel % g.thread_y)
+        return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: thread factors must divide the %dx%d tile (PAPER.md:237)", panel, panel);
+    if (g.flags & RODINIA_STREAM) return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: no stream family");
+    pl->p = panel;
+    pl->v = find(panel, g.thread_x, g.thread_y, g.index_mode);
+    if (!pl->v) return set_error(RODINIA_E_NOT_BUILT, "lud: internal variant P=%d %s not instantiated", panel, gran_str(g).c_str());
+    pl->bx = g.block_x;
+    pl->by = g.block_y;
+    pl->smem = (size_t)(g.block_x + g.block_y) * panel * (panel + 1) * sizeof(float);
+    if (pl->smem > 227 * 1024)
+        return set_error(RODINIA_E_SMEM, "lud: block factor (%d,%d) needs %zu B shared memory > 227 KB (PAPER.md:251)",
+                         g.block_x, g.block_y, pl->smem);
+    return RODINIA_OK;
+}
+
+static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
+    const int P = pl.p, m = (n + P - 1) / P;
+    DPFn diag = P == 16 ? (DPFn)lud_diag<16> : (DPFn)lud_diag<32>;
+    DPFn perim = P == 16 ? (DPFn)lud_perim<16> : (DPFn)lud_perim<32>;
+    for (int k = 0; k < m; ++k) {
+        diag<<<1, P, 0, s>>>(slot, n, k);
+        if (k == m - 1) break;
+        perim<<<m - k - 1, 2 * P, 0, s>>>(slot, n, k);
+        const int rem = m - k - 1;
+        dim3 grid((rem + pl.bx - 1) / pl.bx, (rem + pl.by - 1) / pl.by);
+        dim3 block(P / pl.v->tx, P / pl.v->ty);
+        pl.v->fn<<<grid, block, pl.smem, s>>>(slot, n, k, pl.bx, pl.by);
+    }
+}
+
+struct GraphEntry {
+    cudaGraphExec_t exec = nullptr;
+    float** slot = nullptr;
+    int launches = 0;
+};
+static std::mutex g_mu;
+static std::map<std::tuple<int, int, int, int, int, int, int, int, int>, GraphEntry> g_graphs;
+
+rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
+    int dev = 0;
+    RG_CUDA(cudaGetDevice(&dev));
+    const auto key = std::make_tuple(dev, n, pl.p, pl.v->tx, pl.v->ty, pl.v->mode, pl.bx, pl.by, 0);
+    std::lock_guard<std::mutex> lk(g_mu);
+    GraphEntry& ge = g_graphs[key];
+    const int m = (n + pl.p - 1) / pl.p;
+    if (!ge.exec) {
+        RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
+        if (pl.smem > 48 * 1024)
+            RG_CUDA(cudaFuncSetAttribute((const void*)pl.v->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
+        cudaStream_t cs;
+        RG_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+        cudaGraph_t graph;
+        RG_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+        launch_all(pl, ge.slot, n, cs);
+        cudaError_t e = cudaStreamEndCapture(cs, &graph);
+        cudaStreamDestroy(cs);
+        if (e != cudaSuccess) return cuda_error(e, "lud graph capture", __FILE__, __LINE__);
+        e = cudaGraphInstantiate(&ge.exec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e != cudaSuccess) { ge.exec = nullptr; return cuda_error(e, "lud graph instantiate", __FILE__, __LINE__); }
+        ge.launches = 3 * m - 2;
+    }
+    lud_set_slot<<<1, 1, 0, s>>>(ge.slot, a);
+    RG_CUDA(cudaGraphLaunch(ge.exec, s));
+    count_launch(ge.launches + 1);
+    return RODINIA_OK;
+}
+
+int num_variants() { return (int)(sizeof(kInternal) / sizeof(kInternal[0])); }
+void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    const auto& v = kInternal[i];
+    *g = gran(v.tx, v.ty, 1, 1, 1, v.mode);
+    *fn = (const void*)v.fn;
+    *key = v.key;
+    *threads = (v.p / v.tx) * (v.p / v.ty);
+}
+
+}  // namespace lud
+
+int lud_num_variants() { return lud::num_variants(); }
+void lud_variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    lud::variant_info(i, g, fn, key, threads);
+}
+
+rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p);
+rodinia_status host_buffer(int i, size_t bytes, void** out);
+
+static rodinia_status lud_validate(const void* a, int64_t n, int32_t panel) {
+    if (!a) return set_error(RODINIA_E_INVALID, "lud: null buffer");
+    if (n < 1 || n > 65535 * 16) return set_error(RODINIA_E_INVALID, "lud: n must be in [1, 1048560]");
+    if (panel < 0) return set_error(RODINIA_E_INVALID, "lud: panel < 0");
+    return RODINIA_OK;
+}
+
+__global__ void lud_fill_k(float* a, int n) {
+    // diagonally dominant synthetic matrix for timing (values do not affect the run time)
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < (int64_t)n * n;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = e / n, j = e - i * n;
+        uint32_t x = (uint32_t)e * 2654435761u;
+        x ^= x >> 13;
+        a[e] = (float)(x & 0xffff) * (1.0f / 65536.0f) + (i == j ? (float)n : 0.0f);
+    }
+}
+
+// Tuner: internal variants (panel 16) x block factors {1,2,4,7,8} x {1,2}.
+rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity* best,
+                        std::vector<rodinia_tune_row>* rows) {
+    const int n = (int)pr.rows;
+    cudaStream_t s;
+    RG_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    float* A = nullptr;
+    if (cudaMalloc(&A, (size_t)n * n * 4) != cudaSuccess) {
+        cudaGetLastError();
+        cudaStreamDestroy(s);
+        return set_error(RODINIA_E_NOMEM, "lud tune: allocation failed");
+    }
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    rodinia_status st = RODINIA_OK;
+    float best_ms = 1e30f;
+    for (int vi = 0; st == RODINIA_OK && vi < lud::num_variants(); ++vi) {
+        rodinia_granularity g0;
+        const void* fn;
+        const char* key;
+        int threads;
+        lud::variant_info(vi, &g0, &fn, &key, &threads);
+        if (lud::kInternal[vi].p != 16) continue;
+        for (int bx : {1, 2, 4, 7, 8})
+            for (int by : {1, 2}) {
+                rodinia_tune_row row;
+                memset(&row, 0, sizeof row);
+                row.g = g0;
+                row.g.block_x = bx;
+                row.g.block_y = by;
+                row.median_ms = -1.f;
+                lud::Plan pl;
+                rodinia_status cs = lud::plan(row.g, 16, &pl);
+                const PtxasStats* ps = find_stats(key);
+                row.regs = ps ? ps->regs : -1;
+                row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
+                row.threads = threads;
+                if (cs == RODINIA_OK) {
+                    row.smem_bytes = (int)pl.smem;
+                    if (pl.smem > 48 * 1024)
+                        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem);
+                    row.ctas_per_sm = ctas_per_sm(fn, threads, pl.smem);
+                    cs = filter_decision(ps, threads, (int)pl.smem, 0);
+                    if (cs == RODINIA_OK && row.ctas_per_sm == 0) cs = RODINIA_E_FILTERED;
+                }
+                if (cs == RODINIA_OK) {
+                    std::vector<float> ts;
+                    for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {
+                        lud_fill_k<<<1184, 256, 0, s>>>(A, n);
+                        cudaEventRecord(e0, s);
+                        cs = lud::run(A, n, pl, s);
+                        cudaEventRecord(e1, s);
+                        if (cudaEventSynchronize(e1) != cudaSuccess)
+                            st = cs = cuda_error(cudaGetLastError(), "lud tune", __FILE__, __LINE__);
+                        float ms = 0;
+                        cudaEventElapsedTime(&ms, e0, e1);
+                        if (r >= 0) ts.push_back(ms);
+                    }
+                    if (cs == RODINIA_OK) {
+                        std::sort(ts.begin(), ts.end());
+                        row.median_ms = ts[ts.size() / 2];
+                        if (row.median_ms < best_ms) { best_ms = row.median_ms; *best = row.g; }
+                    }
+                }
+                row.status = cs;
+                rows->push_back(row);
+            }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(A);
+    cudaStreamDestroy(s);
+    if (st == RODINIA_OK && best_ms >= 1e29f) st = set_error(RODINIA_E_FILTERED, "lud tune: no variant survived");
+    if (st == RODINIA_OK) tune_cache_store(RODINIA_LUD, pr, *best, best_ms);
+    return st;
+}
+
+}  // namespace rg
+
+using namespace rg;
+
+extern "C" rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const rodinia_granularity* g, void* stream) {
+    RG_TRY(lud_validate(a, n, panel));
+    rodinia_granularity gg;
+    if (!gran_is_zero(g)) gg = *g;
+    else {
+        rodinia_problem pb{n, n, 1, 1};
+        if (!tune_cache_lookup(RODINIA_LUD, pb, &gg)) gg = default_gran(RODINIA_LUD, pb);
+    }
+    lud::Plan pl;
+    RG_TRY(lud::plan(gg, panel, &pl));
+    DeviceInfo di;
+    RG_TRY(device_info(&di));
+    return lud::run(a, (int)n, pl, (cudaStream_t)stream);
+}
+
+extern "C" rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
+                                           void* stream) {
+    RG_TRY(lud_validate(a, n, panel));
+    DeviceInfo di;
+    RG_TRY(device_info(&di));
+    void* da;
+    RG_TRY(host_buffer(0, (size_t)n * n * 4, &da));
+    cudaStream_t s = (cudaStream_t)stream;
+    RG_CUDA(cudaMemcpyAsync(da, a, (size_t)n * n * 4, cudaMemcpyHostToDevice, s));
+    RG_TRY(rodinia_lud((float*)da, n, panel, g, stream));
+    RG_CUDA(cudaMemcpyAsync(a, da, (size_t)n * n * 4, cudaMemcpyDeviceToHost, s));
+    RG_CUDA(cudaStreamSynchronize(s));
+    return RODINIA_OK;
+}

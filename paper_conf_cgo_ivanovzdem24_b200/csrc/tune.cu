@@ -92,9 +92,9 @@ static int family_base_spill(rodinia_kernel k) {
 rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
     switch (k) {
         case RODINIA_HOTSPOT:
-            // B200 default: streaming temporal blocking, 4 columns per lane,
-            // 8 steps per launch, 4 warps per CTA, 256-row chunks.
-            if (p.iterations >= 8 && p.cols >= 128) return gran(4, 1, 4, 16, 8, 1, RODINIA_STREAM);
+            // B200 default (measured on 16384^2): streaming temporal blocking,
+            // 4 columns per lane, 4 steps per launch, 1 band per CTA, 64-row chunks.
+            if (p.iterations >= 4 && p.cols >= 128) return gran(4, 1, 1, 4, 4, 1, RODINIA_STREAM);
             return gran(4, 1, 1, 1, 1, 1);
         case RODINIA_SRAD: return gran(4, 1, 1, 1, 1, 1);
         case RODINIA_PATHFINDER: return gran(4, 1, 1, 1, 8, 1);
@@ -118,8 +118,11 @@ static rodinia_status fill(float* a, int64_t n, float base, float scale, uint32_
     return RODINIA_OK;
 }
 
-// Candidate granularities to time for hotspot (each combined with the instantiated variants).
-static void hotspot_candidates(const rodinia_problem& p, std::vector<rodinia_granularity>* out) {
+// Candidate granularities for hotspot, two stages (DESIGN.md §5 "TDO"):
+//  stage 1: every instantiation with its base block factors;
+//  stage 2: the 4 fastest instantiations of stage 1 with a sweep of block factors (any
+//           integer is legal; primes included on purpose).
+static void hotspot_stage1(std::vector<rodinia_granularity>* out) {
     const int n = hotspot::num_variants();
     for (int i = 0; i < n; ++i) {
         rodinia_granularity g;
@@ -128,22 +131,29 @@ static void hotspot_candidates(const rodinia_problem& p, std::vector<rodinia_gra
         int threads;
         hotspot::variant_info(i, &g, &fn, &key, &threads);
         if (g.flags & RODINIA_STREAM) {
-            for (int w : {2, 4, 8})
-                for (int by : {8, 16, 32}) {
-                    g.block_x = w;
-                    g.block_y = by;
-                    out->push_back(g);
-                }
+            g.block_x = 1; g.block_y = 4; out->push_back(g);
+            g.block_y = 8; out->push_back(g);
         } else {
-            static const int bxy[][2] = {{1, 1}, {2, 1}, {4, 1}, {1, 2}, {2, 2}, {7, 1}, {8, 1}, {4, 4}};
-            for (auto& b : bxy) {
-                g.block_x = b[0];
-                g.block_y = b[1];
-                out->push_back(g);
-            }
+            g.block_x = 1; g.block_y = 1; out->push_back(g);
+            g.block_x = 2; out->push_back(g);
         }
     }
-    (void)p;
+}
+
+static void hotspot_stage2(const rodinia_granularity& base, std::vector<rodinia_granularity>* out) {
+    rodinia_granularity g = base;
+    if (g.flags & RODINIA_STREAM) {
+        for (int bx : {1, 2})
+            for (int by : {2, 3, 4, 6, 8, 16}) { g.block_x = bx; g.block_y = by; out->push_back(g); }
+    } else {
+        static const int bxy[][2] = {{1, 1}, {2, 1}, {3, 1}, {4, 1}, {7, 1}, {1, 2}, {2, 2}, {4, 4}};
+        for (auto& b : bxy) { g.block_x = b[0]; g.block_y = b[1]; out->push_back(g); }
+    }
+}
+
+static bool same_instantiation(const rodinia_granularity& a, const rodinia_granularity& b) {
+    return a.thread_x == b.thread_x && a.thread_y == b.thread_y && a.temporal == b.temporal &&
+           a.index_mode == b.index_mode && a.flags == b.flags;
 }
 
 static float median(std::vector<float> v) {
@@ -154,7 +164,7 @@ static float median(std::vector<float> v) {
 static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_granularity* best,
                                    std::vector<rodinia_tune_row>* rows) {
     const int64_t R = p.rows, C = p.cols;
-    const int iters = std::max(1, std::min(p.iterations, 48));
+    const int iters = std::max(1, std::min(p.iterations, 24));
     cudaStream_t s;
     RG_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     float *tin = nullptr, *pw = nullptr, *tout = nullptr, *scr = nullptr;
@@ -173,20 +183,17 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
     rodinia_hotspot_coeffs cc;
     rodinia_hotspot_coeffs_rodinia(R, C, R * 31.25e-6, C * 31.25e-6, &cc);
     const HsCoef cf{cc.k, cc.rx, cc.ry, cc.rz, cc.amb};
-    std::vector<rodinia_granularity> cands;
-    hotspot_candidates(p, &cands);
     const int base_spill = family_base_spill(RODINIA_HOTSPOT);
     float best_ms = 1e30f;
-    for (size_t ci = 0; st == RODINIA_OK && ci < cands.size(); ++ci) {
+    auto time_one = [&](const rodinia_granularity& gc) {
         rodinia_tune_row row;
         memset(&row, 0, sizeof row);
-        row.g = cands[ci];
+        row.g = gc;
         row.median_ms = -1.f;
         const hotspot::DirectVariant* dv;
         const hotspot::StreamVariant* sv;
         rodinia_status cs = hotspot::check(row.g, R, C, &dv, &sv);
         if (cs == RODINIA_OK) {
-            // ptxas statistics / filter of the underlying instantiation
             const int n = hotspot::num_variants();
             for (int i = 0; i < n; ++i) {
                 rodinia_granularity g;
@@ -194,11 +201,8 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
                 const char* key;
                 int threads;
                 hotspot::variant_info(i, &g, &fn, &key, &threads);
-                if (g.thread_x == row.g.thread_x && g.thread_y == row.g.thread_y &&
-                    g.temporal == row.g.temporal && g.index_mode == row.g.index_mode &&
-                    (g.flags & RODINIA_STREAM) == (row.g.flags & RODINIA_STREAM)) {
+                if (same_instantiation(g, row.g)) {
                     const PtxasStats* ps = find_stats(key);
-                    if (g.flags & RODINIA_STREAM) threads = 32 * row.g.block_x;
                     row.regs = ps ? ps->regs : -1;
                     row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
                     row.smem_bytes = ps ? ps->smem : -1;
@@ -231,6 +235,29 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
         }
         row.status = cs;
         rows->push_back(row);
+    };
+    std::vector<rodinia_granularity> stage1;
+    hotspot_stage1(&stage1);
+    for (size_t i = 0; st == RODINIA_OK && i < stage1.size(); ++i) time_one(stage1[i]);
+    // stage 2: best 4 distinct instantiations
+    std::vector<rodinia_tune_row> ok;
+    for (auto& r : *rows) if (r.status == RODINIA_OK && r.median_ms > 0) ok.push_back(r);
+    std::sort(ok.begin(), ok.end(), [](const rodinia_tune_row& a, const rodinia_tune_row& b) { return a.median_ms < b.median_ms; });
+    std::vector<rodinia_granularity> tops;
+    for (auto& r : ok) {
+        bool dup = false;
+        for (auto& t : tops) dup = dup || same_instantiation(t, r.g);
+        if (!dup) tops.push_back(r.g);
+        if (tops.size() == 4) break;
+    }
+    for (auto& t : tops) {
+        std::vector<rodinia_granularity> stage2;
+        hotspot_stage2(t, &stage2);
+        for (auto& g : stage2) {
+            bool seen = false;
+            for (auto& r : *rows) seen = seen || (memcmp(&r.g, &g, sizeof g) == 0);
+            if (!seen && st == RODINIA_OK) time_one(g);
+        }
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);

@@ -71,11 +71,15 @@ def _direct_grans():
     return out
 
 
-def _stream_grans():
+def _stream_grans(rg):
+    # every instantiated stream variant that survives the compile-time filter
     out = []
-    for v, h in [(4, 2), (4, 4), (4, 6), (4, 8), (4, 12), (2, 4), (2, 8), (1, 4), (1, 8)]:
-        for w, by in [(1, 1), (4, 3), (8, 16)]:
-            out.append((v, 1, w, by, h, 1, 2))
+    for r in rg.rodinia_variants("hotspot"):
+        g = r["g"]
+        if not (g[6] & rg.RODINIA_STREAM) or r["status"] != 0:
+            continue
+        for bx, by in [(1, 1), (3, 2), (2, 16)]:
+            out.append((g[0], 1, bx, by, g[4], 1, g[6]))
     return out
 
 
@@ -86,7 +90,7 @@ def test_all_variants_bit_identical(rg, R, C):
     iters = 17  # not a multiple of any temporal depth: exercises the remainder launches
     base = _run(rg, T, P, iters, coef, UNC)
     assert rel_err(base, oracle.hotspot(T, P, iters, **coef)) <= TOL
-    for g in _direct_grans() + _stream_grans():
+    for g in _direct_grans() + _stream_grans(rg):
         got = _run(rg, T, P, iters, coef, g)
         assert np.array_equal(got, base), g
 

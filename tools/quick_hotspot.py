@@ -15,10 +15,12 @@ grans = []
 if which in ("all", "direct"):
     grans += [(1,1,1,1,1,0,0), (4,1,1,1,1,1,0), (4,1,2,1,1,1,0), (4,1,4,1,1,1,0), (4,2,2,1,1,1,0), (4,1,2,2,1,1,0)]
 if which in ("all", "stream"):
-    for v, h in [(4,2),(4,4),(4,6),(4,8),(2,4),(2,8),(1,4),(1,8)]:
-        for bx in (1, 2):
-            for by in (4, 8, 16, 32):
-                grans.append((v,1,bx,by,h,1,2))
+    for r in rg.rodinia_variants("hotspot"):
+        g = r["g"]
+        if not (g[6] & 2) or r["status"] != 0:
+            continue
+        for by in (2, 4, 8):
+            grans.append((g[0], 1, 1, by, g[4], 1, g[6]))
 res = []
 for g in grans:
     try:
