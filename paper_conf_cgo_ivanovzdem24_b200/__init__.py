@@ -339,3 +339,6 @@ def rodinia_slab(global_rows: int, nranks: int, rank: int):
           "rodinia_slab")
     return r0.value, n.value
 
+
+
+from . import dist  # noqa: E402  (row-slab multi-GPU layer)

@@ -420,6 +420,8 @@ rodinia_status run(const float* tin, const float* p, float* tout, float* scr, in
 
 int num_variants() { return (int)(sizeof(kDirect) / sizeof(kDirect[0]) + sizeof(kStream) / sizeof(kStream[0])); }
 
+int temporal_of(const StreamVariant* sv) { return sv ? sv->h : 1; }
+
 // Describe variant i: granularity (block factors 1), kernel pointer, key, threads per CTA.
 void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
     const int nd = (int)(sizeof(kDirect) / sizeof(kDirect[0]));

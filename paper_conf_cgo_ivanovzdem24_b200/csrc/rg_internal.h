@@ -75,6 +75,12 @@ inline rodinia_granularity gran(int tx, int ty, int bx, int by, int h, int mode,
 }
 std::string gran_str(const rodinia_granularity& g);
 
+// Default granularity per workload when neither the caller nor the tune cache chooses one.
+rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p);
+
+// Cached device buffers of the *_host entry points (index 0..2), grown on demand.
+rodinia_status host_buffer(int i, size_t bytes, void** out);
+
 // ------------------------------------------------------------------ tune cache
 bool tune_cache_lookup(rodinia_kernel k, const rodinia_problem& p, rodinia_granularity* out);
 void tune_cache_store(rodinia_kernel k, const rodinia_problem& p, const rodinia_granularity& g,

@@ -1,0 +1,107 @@
+"""Row-slab multi-GPU layer (hotspot, srad): thin binding over rodinia_comm_* / *_dist.
+
+One process per GPU.  `HaloComm.from_process_group()` bootstraps the library-owned NCCL
+communicator from a torch.distributed process group (rank 0 creates the NCCL unique id,
+broadcast_object_list ships it); the halo exchange itself runs inside the library
+(ncclSend/ncclRecv on the compute stream).  `HaloComm.local(P)` keeps P slabs
+on the current device (cudaMemcpyAsync halos) to exercise the same slab logic on one GPU.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import (HotspotCoeffs, _dev, _g, _stream, check, lib)
+
+
+def _nccl_path():
+    """Point the library at the libnccl.so.2 torch uses (never the system copy)."""
+    if os.environ.get("RODINIA_NCCL_LIB"):
+        return os.environ["RODINIA_NCCL_LIB"]
+    try:
+        import nvidia.nccl
+        p = os.path.join(list(nvidia.nccl.__path__)[0], "lib", "libnccl.so.2")
+        if os.path.exists(p):
+            os.environ["RODINIA_NCCL_LIB"] = p
+            return p
+    except Exception:
+        pass
+    return None
+
+
+def unique_id() -> bytes:
+    _nccl_path()
+    buf = ctypes.create_string_buffer(128)
+    check(lib.rodinia_comm_unique_id(buf), "rodinia_comm_unique_id")
+    return buf.raw
+
+
+def slab(global_rows: int, nranks: int, rank: int):
+    r0, n = ctypes.c_int64(0), ctypes.c_int64(0)
+    check(lib.rodinia_slab(global_rows, nranks, rank, ctypes.byref(r0), ctypes.byref(n)), "rodinia_slab")
+    return r0.value, n.value
+
+
+class HaloComm:
+    def __init__(self, handle, nranks: int, rank: int, local: bool):
+        self.handle = handle
+        self.nranks = nranks
+        self.rank = rank
+        self.local = local
+
+    @classmethod
+    def from_process_group(cls, group=None):
+        import torch.distributed as dist
+        ws, rank = dist.get_world_size(group), dist.get_rank(group)
+        obj = [unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        h = ctypes.c_void_p()
+        _nccl_path()
+        check(lib.rodinia_comm_init(ctypes.byref(h), ws, rank, obj[0]), "rodinia_comm_init")
+        return cls(h, ws, rank, local=False)
+
+    @classmethod
+    def local_slabs(cls, nranks: int):
+        h = ctypes.c_void_p()
+        check(lib.rodinia_comm_init_local(ctypes.byref(h), nranks), "rodinia_comm_init_local")
+        return cls(h, nranks, 0, local=True)
+
+    def close(self):
+        if self.handle:
+            check(lib.rodinia_comm_destroy(self.handle), "rodinia_comm_destroy")
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------------ marshalling
+    def _ptrs(self, x, dtype, name):
+        if self.local:
+            arr = (ctypes.c_void_p * self.nranks)(*[_dev(t, dtype, name).value for t in x])
+            return ctypes.cast(arr, ctypes.c_void_p), arr
+        return _dev(x, dtype, name), None
+
+    def hotspot(self, temp_local, power_local, out_local, global_rows: int, iterations: int,
+                coeffs: HotspotCoeffs | None = None, g=None, stream=None):
+        """One rank's slab (or, for a local communicator, lists of all slabs)."""
+        import torch
+        t, keep1 = self._ptrs(temp_local, torch.float32, "temp")
+        p, keep2 = self._ptrs(power_local, torch.float32, "power")
+        o, keep3 = self._ptrs(out_local, torch.float32, "out")
+        cols = (temp_local[0] if self.local else temp_local).shape[1]
+        check(lib.rodinia_hotspot_dist(self.handle, t, p, o, global_rows, cols, int(iterations),
+                                       None if coeffs is None else ctypes.byref(coeffs), _g(g),
+                                       _stream(stream)), "rodinia_hotspot_dist")
+        return out_local
+
+    def srad(self, J_local, global_rows: int, r1, r2, c1, c2, lam: float, niter: int, g=None,
+             stream=None):
+        import torch
+        j, keep = self._ptrs(J_local, torch.float32, "J")
+        cols = (J_local[0] if self.local else J_local).shape[1]
+        check(lib.rodinia_srad_dist(self.handle, j, global_rows, cols, r1, r2, c1, c2, float(lam),
+                                    int(niter), _g(g), _stream(stream)), "rodinia_srad_dist")
+        return J_local
