@@ -86,13 +86,13 @@ def test_ptxas_parser_on_canned_log():
     text = open(os.path.join(ROOT, "tests", "golden", "ptxas_sample.log")).read()
     st = ptxas_filter.parse_ptxas_log(text)
     assert set(s.key for s in st.values()) == {
-        "void rg::hs_direct<16, 2, 1>", "void rg::hs_direct<1, 1, 0>", "big_smem()"}
+        "void rg::hs_direct<16, 2, 1>", "void rg::hs_direct<1, 1, 0>", "big_smem"}
     by = {s.key: s for s in st.values()}
     a = by["void rg::hs_direct<16, 2, 1>"]
     assert (a.regs, a.spill_stores, a.spill_loads, a.stack) == (64, 8, 12, 8)
     b = by["void rg::hs_direct<1, 1, 0>"]
     assert (b.regs, b.spill_stores, b.spill_loads) == (40, 0, 0)
-    assert by["big_smem()"].smem == 233472
+    assert by["big_smem"].smem == 233472
 
 
 def test_prune_rules():
