@@ -294,7 +294,10 @@ def run_ours(args):
 
     # ---- tuning (TDO) on synthetic data of the problem's shape, before the timed region
     t_tune = time.perf_counter()
-    if args.no_tune:
+    if args.gran:
+        g = rg.gran(*[int(x) for x in args.gran.split(",")])
+        tune_rows = []
+    elif args.no_tune:
         g = rg.rodinia_resolve("hotspot", N, N, iters, ws)
         tune_rows = []
     else:
@@ -439,6 +442,7 @@ def main():
     ap.add_argument("--no-tune", action="store_true")
     ap.add_argument("--no-extra", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--gran", type=str, default="", help="fixed hotspot granularity tx,ty,bx,by,h,mode,flags")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

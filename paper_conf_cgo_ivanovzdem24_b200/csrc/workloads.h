@@ -32,10 +32,13 @@ struct SradIter {       // written by srad_roi_stats, read by the pass kernels
 namespace srad {
 typedef void (*FusedFn)(const float*, float*, int, int, int, int, float, const SradIter*);
 struct Variant { int tx, ty, mode; FusedFn fn; const char* key; };
+typedef void (*StreamFn)(const float*, float*, int, int, int, int, float, const SradIter*, int);
+struct StreamVariant { int v; StreamFn fn; const char* key; };
 // Plan: dataflow (uncoarsened) iff granularity is exactly the uncoarsened one.
 struct Plan {
     bool dataflow;
     const Variant* v;
+    const StreamVariant* stream;   // stream family (flags & RODINIA_STREAM)
     int bx, by;
     size_t smem;
 };

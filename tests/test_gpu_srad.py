@@ -40,7 +40,7 @@ def test_vs_oracle(rg, R, C):
     roi = _roi(R, C)
     for n in (1, 5, 20):
         ref = oracle.srad(J, *roi, 0.5, n)
-        for g in (UNC, (4, 1, 2, 2, 1, 1, 0)):
+        for g in (UNC, (4, 1, 2, 2, 1, 1, 0), (4, 1, 1, 2, 1, 1, 2)):
             got = _run(rg, J, roi, 0.5, n, g)
             assert rel_err(got, ref) <= TOL, (R, C, n, g, rel_err(got, ref))
 
@@ -64,12 +64,24 @@ def _fused_grans():
     return out
 
 
-def test_all_variants_bit_identical(rg):
-    J = synth.srad_input(131, 97, seed=3)
-    roi = (0, 60, 5, 70)
+def _stream_grans(rg):
+    out = []
+    for r in rg.rodinia_variants("srad"):
+        g = r["g"]
+        if (g[6] & rg.RODINIA_STREAM) and r["status"] == 0:
+            for bx, by in [(1, 1), (2, 3), (1, 8)]:
+                out.append((g[0], 1, bx, by, 1, 1, g[6]))
+    assert out
+    return out
+
+
+@pytest.mark.parametrize("R,C", [(131, 97), (70, 256), (33, 260)])
+def test_all_variants_bit_identical(rg, R, C):
+    J = synth.srad_input(R, C, seed=3)
+    roi = (0, min(60, R - 1), 5, 70)
     base = _run(rg, J, roi, 0.5, 6, UNC)
     assert rel_err(base, oracle.srad(J, *roi, 0.5, 6)) <= TOL
-    for g in _fused_grans():
+    for g in _fused_grans() + _stream_grans(rg):
         assert np.array_equal(_run(rg, J, roi, 0.5, 6, g), base), g
 
 
