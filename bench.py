@@ -344,11 +344,16 @@ def run_ours(args):
     avg_launch_ms = ms / max(launches_per_step, 1)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "r01_hotspot_traffic.json")
-    if os.path.exists(tp):
+    # DRAM traffic per launch from the committed ncu --set full capture of the same kernel and
+    # granularity (profiles/<round>_hotspot.json), newest round first
+    import glob
+    for tp in sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_hotspot.json")), reverse=True):
         try:
             with open(tp) as f:
-                traffic = json.load(f).get("traffic_bytes_per_launch")
+                prof = json.load(f)
+            if prof.get("granularity") == list(g.astuple()) and prof.get("traffic_bytes_per_launch"):
+                traffic = prof["traffic_bytes_per_launch"] * (rows_local * N) / (16384 * 16384)
+                break
         except Exception:
             traffic = None
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",

@@ -136,20 +136,29 @@ __device__ __forceinline__ void hs_ld(const float* __restrict__ base, int row, i
     }
 }
 
+// Loads are prefetched three rows ahead (register queues tq/pq, period 3 like the rings).  The
+// power row consumed by level 1 is parked in a per-warp shared-memory ring of H rows from which
+// levels 2..H read it back in later steps (each lane reads only its own columns, so no
+// synchronisation is needed); this replaces H-1 global re-loads per step.
 template <int V, int H, int K, bool EC, bool ER>
-__device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&nxt_t)[V],
-                                               float (&nxt_p)[V], const float* __restrict__ tin,
+__device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&tq)[3][V], float (&pq)[3][V],
+                                               float* __restrict__ psm, const float* __restrict__ tin,
                                                const float* __restrict__ pw, float* __restrict__ tout,
-                                               int g0, int R, int C, int ylo, int yhi, int sc0, int col0,
+                                               int s, int g0, int R, int C, int ylo, int yhi, int sc0, int col0,
                                                const HsCoef& cf) {
     constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
-    // level 0: the prefetched row g0 becomes the newest level-0 row; prefetch T row g0+1 and the
-    // power row g0 (needed by level 1 at the next step).
+    // level 0 takes T row g0; level 1 takes P row g0-1; refill both queues three rows ahead
     float p1[V];
 #pragma unroll
-    for (int v = 0; v < V; ++v) { ring[0][S2][v] = nxt_t[v]; p1[v] = nxt_p[v]; }
-    hs_ld<V, EC, ER>(tin, g0 + 1, R, C, col0, nxt_t);
-    hs_ld<V, EC, ER>(pw, g0, R, C, col0, nxt_p);
+    for (int v = 0; v < V; ++v) { ring[0][S2][v] = tq[K][v]; p1[v] = pq[K][v]; }
+    hs_ld<V, EC, ER>(tin, g0 + 3, R, C, col0, tq[K]);
+    hs_ld<V, EC, ER>(pw, g0 + 2, R, C, col0, pq[K]);
+    const int sb = s % H;
+    if (H > 1) {
+        float* dst = psm + (sb * 32 * V) + sc0;
+#pragma unroll
+        for (int v = 0; v < V; ++v) dst[v] = p1[v];
+    }
 
 #pragma unroll
     for (int l = 0; l < H; ++l) {
@@ -159,7 +168,11 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&n
 #pragma unroll
             for (int v = 0; v < V; ++v) pv[v] = p1[v];
         } else {
-            hs_ld<V, EC, ER>(pw, g, R, C, col0, pv);  // L1 hit: first touched by level 1
+            int slot = sb + H - l;
+            slot -= (slot >= H) ? H : 0;
+            const float* src = psm + slot * 32 * V + sc0;
+#pragma unroll
+            for (int v = 0; v < V; ++v) pv[v] = src[v];
         }
         const bool top = ER && (g == 0), bot = ER && (g == R - 1);
         const float wnb = __shfl_up_sync(0xffffffffu, ring[l][S1][V - 1], 1);
@@ -169,7 +182,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&n
         for (int v = 0; v < V; ++v) {
             const float c = ring[l][S1][v];
             const float n = top ? c : ring[l][S0][v];
-            const float s = bot ? c : ring[l][S2][v];
+            const float s_ = bot ? c : ring[l][S2][v];
             float w = v > 0 ? ring[l][S1][v > 0 ? v - 1 : 0] : wnb;
             float e = v < V - 1 ? ring[l][S1][v < V - 1 ? v + 1 : 0] : enb;
             if (EC) {
@@ -177,7 +190,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&n
                 if (col == 0) w = c;
                 if (col == C - 1) e = c;
             }
-            res[v] = hs_cell(c, n, s, e, w, pv[v], cf);
+            res[v] = hs_cell(c, n, s_, e, w, pv[v], cf);
         }
         if (l + 1 < H) {
 #pragma unroll
@@ -208,8 +221,8 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&n
 template <int V, int H, bool EC, bool ER>
 __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
                                                const float* __restrict__ pw,
-                                               float* __restrict__ tout, int R, int C, int y0,
-                                               int y1, int sc0, int col0, const HsCoef& cf) {
+                                               float* __restrict__ tout, float* __restrict__ psm, int R,
+                                               int C, int y0, int y1, int sc0, int col0, const HsCoef& cf) {
     float ring[H][3][V];
 #pragma unroll
     for (int l = 0; l < H; ++l)
@@ -219,17 +232,20 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
             for (int v = 0; v < V; ++v) ring[l][k][v] = 0.0f;
     const int ystart = y0 - H;
     const int nsteps = (y1 - y0) + 2 * H;
-    float nxt_t[V], nxt_p[V];
-    hs_ld<V, EC, ER>(tin, ystart, R, C, col0, nxt_t);
-    hs_ld<V, EC, ER>(pw, ystart - 1, R, C, col0, nxt_p);
+    float tq[3][V], pq[3][V];
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+        hs_ld<V, EC, ER>(tin, ystart + k, R, C, col0, tq[k]);
+        hs_ld<V, EC, ER>(pw, ystart - 1 + k, R, C, col0, pq[k]);
+    }
     int s = 0;
     for (; s + 3 <= nsteps; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 1, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 2, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 2, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 0, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s, ystart + s, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 1, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 1, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 2, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 2, ystart + s + 2, R, C, y0, y1, sc0, col0, cf);
     }
-    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s, R, C, y0, y1, sc0, col0, cf);
-    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, nxt_t, nxt_p, tin, pw, tout, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s, ystart + s, R, C, y0, y1, sc0, col0, cf);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 1, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
 }
 
 // One warp per CTA: every branch condition derives from blockIdx and kernel arguments only, so
@@ -247,7 +263,9 @@ __global__ void __launch_bounds__(32, OCC)
     const int sc0 = (int)threadIdx.x * V;
     const int y0 = blockIdx.y * chunk;
     const int y1 = min(y0 + chunk, R);
-    const bool er = (y0 - H - 1 < 0) || (y1 + H > R - 1);
+    // rows touched: T [y0-H, y1+H+2], P [y0-H-1, y1+H+1] (prefetch queues run 3 rows ahead)
+    const bool er = (y0 - H - 1 < 0) || (y1 + H + 2 > R - 1);
+    __shared__ __align__(16) float psm[H * 32 * V];
     for (int bi = 0; bi < bands_per_cta; ++bi) {
         const int band = blockIdx.x * bands_per_cta + bi;
         if (band * OW >= C) return;
@@ -255,13 +273,13 @@ __global__ void __launch_bounds__(32, OCC)
         const int col0 = bstart + sc0;
         const bool ec = !vec_ok || bstart < 0 || bstart + SW > C;
         if (!ec && !er)
-            hs_stream_body<V, H, false, false>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, false, false>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
         else if (ec && !er)
-            hs_stream_body<V, H, true, false>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, true, false>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
         else if (!ec && er)
-            hs_stream_body<V, H, false, true>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, false, true>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
         else
-            hs_stream_body<V, H, true, true>(tin, pw, tout, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, true, true>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
     }
 }
 

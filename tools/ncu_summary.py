@@ -67,9 +67,10 @@ def main():
     ap.add_argument("--rep")
     ap.add_argument("--out", required=True)
     ap.add_argument("--algo-bytes", type=float, default=None)
+    ap.add_argument("--gran", default="", help="granularity the capture was taken with")
     a = ap.parse_args()
-    res = {}
-    md = []
+    res = {"granularity": [int(x) for x in a.gran.split(",")] if a.gran else None}
+    md = [f"granularity: {a.gran}\n"] if a.gran else []
     if a.launches:
         L = launches(a.launches)
         res["launch_list"] = L

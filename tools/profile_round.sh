@@ -1,0 +1,13 @@
+#!/bin/bash
+# One GPU session: bench (tuned), then the ncu launch list and a --set full capture of the
+# dominant kernel with the bench's tuned granularity.  Outputs under gpurun_out/.
+set -x
+TAG=${1:-r01}
+python bench.py > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
+G=$(python -c "import json;print(','.join(map(str,json.load(open('gpurun_out/bench_${TAG}.json'))['config']['granularity'])))")
+echo "tuned granularity: $G"
+ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file gpurun_out/launches_${TAG}.csv \
+    python bench.py --steps 1 --warmup 3 --gran $G --no-extra --no-cpu > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:hs_ -s 12 -c 1 -o gpurun_out/prof_${TAG}_hotspot \
+    python bench.py --steps 1 --warmup 3 --gran $G --no-extra --no-cpu --iters 48 > gpurun_out/ncu_${TAG}.log 2>&1
+tail -2 gpurun_out/ncu_${TAG}.log
