@@ -32,133 +32,209 @@
 namespace rg {
 
 // ------------------------------------------------------------------ diagonal tile
+// One warp.  Lane i holds row i of the tile in registers; step k broadcasts row k with warp
+// shuffles and every lane below it subtracts l_ik * u_kj.  Per element this is exactly
+// Doolittle's sequence (products subtracted in ascending k, L divided by the pivot after its
+// k < j terms), computed with separate multiply and subtract as in Rodinia's lud_diagonal.
 template <int P>
-__global__ void __launch_bounds__(P) lud_diag(float* const* __restrict__ slot, int n, int k) {
+__global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, int n, int k) {
     float* A = *slot;
-    __shared__ float t[P][P + 1];
-    const int o = k * P, r = min(P, n - o), tx = threadIdx.x;
-    for (int i = 0; i < r; ++i)
-        if (tx < r) t[i][tx] = A[(size_t)(o + i) * n + o + tx];
-    __syncthreads();
-    for (int i = 0; i < r - 1; ++i) {
-        if (tx > i && tx < r) {  // column i of L
-            float v = t[tx][i];
-            for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(t[tx][j], t[j][i]));
-            t[tx][i] = __fdiv_rn(v, t[i][i]);
+    const int o = k * P, r = min(P, n - o), lane = threadIdx.x;
+    float a[P];
+    const bool own = lane < r;
+#pragma unroll
+    for (int j = 0; j < P; ++j) a[j] = (own && j < r) ? A[(size_t)(o + lane) * n + o + j] : 0.f;
+#pragma unroll
+    for (int kk = 0; kk < P - 1; ++kk) {
+        if (kk >= r - 1) break;  // uniform
+        const float piv = __shfl_sync(0xffffffffu, a[kk], kk);
+        const bool below = lane > kk && own;
+        const float l = __fdiv_rn(a[kk], piv);
+        if (below) a[kk] = l;
+#pragma unroll
+        for (int j = kk + 1; j < P; ++j) {
+            const float ukj = __shfl_sync(0xffffffffu, a[j], kk);
+            if (below) a[j] = __fsub_rn(a[j], __fmul_rn(l, ukj));
         }
-        __syncthreads();
-        if (tx > i && tx < r) {  // row i+1 of U
-            float v = t[i + 1][tx];
-            for (int j = 0; j < i + 1; ++j) v = __fsub_rn(v, __fmul_rn(t[i + 1][j], t[j][tx]));
-            t[i + 1][tx] = v;
-        }
-        __syncthreads();
     }
-    for (int i = 0; i < r; ++i)
-        if (tx < r) A[(size_t)(o + i) * n + o + tx] = t[i][tx];
+#pragma unroll
+    for (int j = 0; j < P; ++j)
+        if (own && j < r) A[(size_t)(o + lane) * n + o + j] = a[j];
 }
 
 // ------------------------------------------------------------------ perimeter tiles
-// CTA j handles the j-th tile right of the diagonal (threads 0..P-1, one column each) and the
-// j-th tile below it (threads P..2P-1, one row each).
+// CTA j handles the j-th tile right of the diagonal and the j-th tile below it: lanes 0..P-1
+// each own one column of U12 = L11^-1 A12 (forward substitution, unit-lower L11), lanes
+// P..2P-1 each own one row of L21 = A21 U11^-1.  Tiles are staged through shared memory with
+// coalesced loads, the substitutions run in registers with L11/U11 read by broadcast.
 template <int P>
 __global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
     float* A = *slot;
-    __shared__ float dia[P][P + 1], row[P][P + 1], col[P][P + 1];
+    __shared__ float dia[P][P + 1], rowt[P][P + 1], colt[P][P + 1];
     const int o = k * P;
-    const int r = P;  // diagonal tile is full whenever perimeter tiles exist
     const int tb = o + P * (blockIdx.x + 1);  // first row/col of this perimeter tile
     const int w = min(P, n - tb);             // its width (last tile may be partial)
     const int tx = threadIdx.x;
-    if (tx < P) {
-        for (int i = 0; i < r; ++i) dia[i][tx] = A[(size_t)(o + i) * n + o + tx];
-        for (int i = 0; i < r; ++i) row[i][tx] = tx < w ? A[(size_t)(o + i) * n + tb + tx] : 0.f;
-    } else {
-        const int c = tx - P;
-        for (int i = 0; i < w; ++i) col[i][c] = A[(size_t)(tb + i) * n + o + c];
+    for (int e = tx; e < P * P; e += 2 * P) {
+        const int i = e / P, j = e % P;
+        dia[i][j] = A[(size_t)(o + i) * n + o + j];
+        rowt[i][j] = j < w ? A[(size_t)(o + i) * n + tb + j] : 0.f;
+        colt[i][j] = i < w ? A[(size_t)(tb + i) * n + o + j] : 0.f;
     }
     __syncthreads();
-    if (tx < P) {
-        if (tx < w)  // U12 column tx: forward substitution with unit-lower L11
-            for (int i = 1; i < r; ++i) {
-                float v = row[i][tx];
-                for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(dia[i][j], row[j][tx]));
-                row[i][tx] = v;
-            }
-    } else {
-        const int idx = tx - P;
-        if (idx < w)  // L21 row idx: solve against U11
-            for (int i = 0; i < r; ++i) {
-                float v = col[idx][i];
-                for (int j = 0; j < i; ++j) v = __fsub_rn(v, __fmul_rn(col[idx][j], dia[j][i]));
-                col[idx][i] = __fdiv_rn(v, dia[i][i]);
-            }
-    }
-    __syncthreads();
-    if (tx < P) {
+    float v[P];
+    if (tx < P) {  // U12 column tx
+#pragma unroll
+        for (int i = 0; i < P; ++i) v[i] = rowt[i][tx];
+#pragma unroll
+        for (int i = 1; i < P; ++i)
+#pragma unroll
+            for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(dia[i][j], v[j]));
         if (tx < w)
-            for (int i = 0; i < r; ++i) A[(size_t)(o + i) * n + tb + tx] = row[i][tx];
-    } else {
-        const int c = tx - P;
-        for (int i = 0; i < w; ++i) A[(size_t)(tb + i) * n + o + c] = col[i][c];
+#pragma unroll
+            for (int i = 0; i < P; ++i) A[(size_t)(o + i) * n + tb + tx] = v[i];
+    } else {  // L21 row idx
+        const int idx = tx - P;
+#pragma unroll
+        for (int i = 0; i < P; ++i) v[i] = colt[idx][i];
+#pragma unroll
+        for (int i = 0; i < P; ++i) {
+#pragma unroll
+            for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(v[j], dia[j][i]));
+            v[i] = __fdiv_rn(v[i], dia[i][i]);
+        }
+        if (idx < w)
+#pragma unroll
+            for (int i = 0; i < P; ++i) A[(size_t)(tb + idx) * n + o + i] = v[i];
     }
 }
 
 // ------------------------------------------------------------------ trailing update
+// The CTA stages by L21 tiles and bx U12 tiles in shared memory and walks its bx*by trailing
+// tiles; each thread's TX x TY elements of the next tile are loaded into registers while the
+// current tile is being updated (software pipelining of the read-modify-write, which is what
+// bounds this kernel by HBM).  MODE 1 with TX % 4 == 0 moves A with 128-bit accesses.
+template <int P, int TX, int TY, int MODE>
+__device__ __forceinline__ void lud_tile_io(float* A, int n, int cx, int cy, float (&av)[TY][TX], bool load) {
+    constexpr int NTX = P / TX, NTY = P / TY;
+#pragma unroll
+    for (int t_y = 0; t_y < TY; ++t_y) {
+        const int ly = MODE == 0 ? (int)threadIdx.y + t_y * NTY : (int)threadIdx.y * TY + t_y;
+        const int gr = cy + ly;
+        if (MODE == 1 && TX % 4 == 0) {
+            const int gc0 = cx + (int)threadIdx.x * TX;
+            if (gr < n && gc0 + TX <= n && (n & 3) == 0) {
+                float4* p = reinterpret_cast<float4*>(A + (size_t)gr * n + gc0);
+#pragma unroll
+                for (int q = 0; q < TX / 4; ++q) {
+                    if (load) {
+                        const float4 t = p[q];
+                        av[t_y][4 * q] = t.x; av[t_y][(4 * q + 1) % TX] = t.y;
+                        av[t_y][(4 * q + 2) % TX] = t.z; av[t_y][(4 * q + 3) % TX] = t.w;
+                    } else {
+                        p[q] = make_float4(av[t_y][4 * q], av[t_y][(4 * q + 1) % TX], av[t_y][(4 * q + 2) % TX],
+                                           av[t_y][(4 * q + 3) % TX]);
+                    }
+                }
+                continue;
+            }
+        }
+#pragma unroll
+        for (int t_x = 0; t_x < TX; ++t_x) {
+            const int lx = MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x;
+            const int gc = cx + lx;
+            if (gr < n && gc < n) {
+                if (load) av[t_y][t_x] = A[(size_t)gr * n + gc];
+                else A[(size_t)gr * n + gc] = av[t_y][t_x];
+            }
+        }
+    }
+}
+
 template <int P, int TX, int TY, int MODE>
 __global__ void __launch_bounds__((P / TX) * (P / TY),
                                   (1024 / ((P / TX) * (P / TY))) < 32 ? (1024 / ((P / TX) * (P / TY))) : 32)
     lud_internal(float* const* __restrict__ slot, int n, int k, int bx, int by) {
     float* A = *slot;
-    extern __shared__ float lsm[];
+    extern __shared__ __align__(16) float lsm[];
     constexpr int NTX = P / TX, NTY = P / TY, NT = NTX * NTY;
+    constexpr int LD = P + 4;  // row pitch of the staged tiles (16-byte aligned rows)
     const int o = k * P;
     const int t0 = o + P;  // first trailing row/col
     const int cx0 = t0 + blockIdx.x * bx * P, cy0 = t0 + blockIdx.y * by * P;
-    float* Ush = lsm;                      // bx tiles of U12: [bx][P][P+1] (rows i, cols)
-    float* Lsh = lsm + bx * P * (P + 1);   // by tiles of L21: [by][P][P+1] (rows, i)
+    float* Ush = lsm;                // bx U12 tiles: Ush[(b*P + i)*LD + c] = U12[i][c]
+    float* Lsh = lsm + bx * P * LD;  // by L21 tiles, transposed: Lsh[(b*P + i)*LD + r] = L21[r][i]
     const int tid = threadIdx.y * NTX + threadIdx.x;
+    float av[TY][TX];
+    lud_tile_io<P, TX, TY, MODE>(A, n, cx0, cy0, av, true);  // first tile's A, before staging
     for (int e = tid; e < bx * P * P; e += NT) {
         const int b = e / (P * P), rem = e - b * P * P, i = rem / P, c = rem - i * P;
         const int gc = cx0 + b * P + c;
-        Ush[(b * P + i) * (P + 1) + c] = gc < n ? A[(size_t)(o + i) * n + gc] : 0.f;
+        Ush[(b * P + i) * LD + c] = gc < n ? A[(size_t)(o + i) * n + gc] : 0.f;
     }
     for (int e = tid; e < by * P * P; e += NT) {
         const int b = e / (P * P), rem = e - b * P * P, rr = rem / P, i = rem - rr * P;
         const int gr = cy0 + b * P + rr;
-        Lsh[(b * P + rr) * (P + 1) + i] = gr < n ? A[(size_t)gr * n + o + i] : 0.f;
+        Lsh[(b * P + i) * LD + rr] = gr < n ? A[(size_t)gr * n + o + i] : 0.f;
     }
     __syncthreads();
-    for (int b_y = 0; b_y < by; ++b_y)
-        for (int b_x = 0; b_x < bx; ++b_x)
+    const int ntiles = bx * by;
+    for (int t = 0; t < ntiles; ++t) {
+        const int b_y = t / bx, b_x = t - b_y * bx;
+        float nx[TY][TX];
+        if (t + 1 < ntiles) {
+            const int n_y = (t + 1) / bx, n_x = (t + 1) - n_y * bx;
+            lud_tile_io<P, TX, TY, MODE>(A, n, cx0 + n_x * P, cy0 + n_y * P, nx, true);
+        }
+        float sum[TY][TX];
 #pragma unroll
-            for (int t_y = 0; t_y < TY; ++t_y) {
-                const int ly = MODE == 0 ? (int)threadIdx.y + t_y * NTY : (int)threadIdx.y * TY + t_y;
-                const int gr = cy0 + b_y * P + ly;
-                float sum[TX];
+        for (int t_y = 0; t_y < TY; ++t_y)
 #pragma unroll
-                for (int t_x = 0; t_x < TX; ++t_x) sum[t_x] = 0.f;
+            for (int t_x = 0; t_x < TX; ++t_x) sum[t_y][t_x] = 0.f;
+        const float* Ub = Ush + (b_x * P) * LD;
+        const float* Lb = Lsh + (b_y * P) * LD;
 #pragma unroll 4
-                for (int i = 0; i < P; ++i) {
-                    const float l = Lsh[(b_y * P + ly) * (P + 1) + i];
+        for (int i = 0; i < P; ++i) {
+            float u[TX], l[TY];
+            if (MODE == 1 && TX % 4 == 0) {
 #pragma unroll
-                    for (int t_x = 0; t_x < TX; ++t_x) {
-                        const int lx = MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x;
-                        sum[t_x] = __fmaf_rn(l, Ush[(b_x * P + i) * (P + 1) + lx], sum[t_x]);
-                    }
+                for (int q = 0; q < TX / 4; ++q) {
+                    const float4 t4 = reinterpret_cast<const float4*>(Ub + i * LD + threadIdx.x * TX)[q];
+                    u[4 * q] = t4.x; u[(4 * q + 1) % TX] = t4.y; u[(4 * q + 2) % TX] = t4.z; u[(4 * q + 3) % TX] = t4.w;
                 }
-                if (gr < n) {
+            } else {
 #pragma unroll
-                    for (int t_x = 0; t_x < TX; ++t_x) {
-                        const int lx = MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x;
-                        const int gc = cx0 + b_x * P + lx;
-                        if (gc < n) {
-                            float* a = A + (size_t)gr * n + gc;
-                            *a = __fsub_rn(*a, sum[t_x]);
-                        }
-                    }
-                }
+                for (int t_x = 0; t_x < TX; ++t_x)
+                    u[t_x] = Ub[i * LD + (MODE == 0 ? (int)threadIdx.x + t_x * NTX : (int)threadIdx.x * TX + t_x)];
             }
+            if (MODE == 1 && TY % 4 == 0) {
+#pragma unroll
+                for (int q = 0; q < TY / 4; ++q) {
+                    const float4 t4 = reinterpret_cast<const float4*>(Lb + i * LD + threadIdx.y * TY)[q];
+                    l[4 * q] = t4.x; l[(4 * q + 1) % TY] = t4.y; l[(4 * q + 2) % TY] = t4.z; l[(4 * q + 3) % TY] = t4.w;
+                }
+            } else {
+#pragma unroll
+                for (int t_y = 0; t_y < TY; ++t_y)
+                    l[t_y] = Lb[i * LD + (MODE == 0 ? (int)threadIdx.y + t_y * NTY : (int)threadIdx.y * TY + t_y)];
+            }
+#pragma unroll
+            for (int t_y = 0; t_y < TY; ++t_y)
+#pragma unroll
+                for (int t_x = 0; t_x < TX; ++t_x) sum[t_y][t_x] = __fmaf_rn(l[t_y], u[t_x], sum[t_y][t_x]);
+        }
+#pragma unroll
+        for (int t_y = 0; t_y < TY; ++t_y)
+#pragma unroll
+            for (int t_x = 0; t_x < TX; ++t_x) av[t_y][t_x] = __fsub_rn(av[t_y][t_x], sum[t_y][t_x]);
+        lud_tile_io<P, TX, TY, MODE>(A, n, cx0 + b_x * P, cy0 + b_y * P, av, false);
+        if (t + 1 < ntiles) {
+#pragma unroll
+            for (int t_y = 0; t_y < TY; ++t_y)
+#pragma unroll
+                for (int t_x = 0; t_x < TX; ++t_x) av[t_y][t_x] = nx[t_y][t_x];
+        }
+    }
 }
 
 __global__ void lud_set_slot(float** slot, float* a) { *slot = a; }
@@ -176,7 +252,8 @@ static const Variant kInternal[] = {
     RG_LI2(16, 1, 4), RG_LI2(16, 4, 2), RG_LI2(16, 2, 4), RG_LI2(16, 4, 4), RG_LI2(16, 8, 1),
     RG_LI2(16, 8, 2), RG_LI2(16, 16, 1), RG_LI2(16, 16, 2),
     RG_LI2(32, 1, 1), RG_LI2(32, 2, 1), RG_LI2(32, 2, 2), RG_LI2(32, 4, 1), RG_LI2(32, 4, 2),
-    RG_LI2(32, 4, 4), RG_LI2(32, 8, 2),
+    RG_LI2(32, 4, 4), RG_LI2(32, 8, 2), RG_LI2(32, 2, 4), RG_LI2(32, 1, 4), RG_LI2(32, 8, 4),
+    RG_LI2(32, 4, 8),
 };
 #undef RG_LI2
 #undef RG_LI
@@ -210,7 +287,7 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
     if (!pl->v) return set_error(RODINIA_E_NOT_BUILT, "lud: internal variant P=%d %s not instantiated", panel, gran_str(g).c_str());
     pl->bx = g.block_x;
     pl->by = g.block_y;
-    pl->smem = (size_t)(g.block_x + g.block_y) * panel * (panel + 1) * sizeof(float);
+    pl->smem = (size_t)(g.block_x + g.block_y) * panel * (panel + 4) * sizeof(float);
     if (pl->smem > 227 * 1024)
         return set_error(RODINIA_E_SMEM, "lud: block factor (%d,%d) needs %zu B shared memory > 227 KB (PAPER.md:251)",
                          g.block_x, g.block_y, pl->smem);
@@ -222,7 +299,7 @@ static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
     DPFn diag = P == 16 ? (DPFn)lud_diag<16> : (DPFn)lud_diag<32>;
     DPFn perim = P == 16 ? (DPFn)lud_perim<16> : (DPFn)lud_perim<32>;
     for (int k = 0; k < m; ++k) {
-        diag<<<1, P, 0, s>>>(slot, n, k);
+        diag<<<1, 32, 0, s>>>(slot, n, k);
         if (k == m - 1) break;
         perim<<<m - k - 1, 2 * P, 0, s>>>(slot, n, k);
         const int rem = m - k - 1;
