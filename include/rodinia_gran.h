@@ -171,7 +171,8 @@ rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel,
  */
 typedef struct {
     int64_t rows, cols;      /* lud: rows = cols = n; pathfinder: rows x cols wall */
-    int32_t iterations;      /* hotspot / srad iterations (tuning times min(iterations, 50)) */
+    int32_t iterations;      /* hotspot / srad iterations (tuning times a prefix of them);
+                                lud: the panel width (0 => 16); pathfinder: unused */
     int32_t nranks;          /* 1 for single-GPU problems; part of the cache key */
 } rodinia_problem;
 

@@ -384,10 +384,12 @@ __global__ void lud_fill_k(float* a, int n) {
     }
 }
 
-// Tuner: internal variants (panel 16) x block factors {1,2,4,7,8} x {1,2}.
+// Tuner: internal variants of the requested panel width x block factors {1,2,4,7} x {1,2,4}.
+// For lud, rodinia_problem.iterations carries the panel width (0 => 16, reading L5).
 rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity* best,
                         std::vector<rodinia_tune_row>* rows) {
     const int n = (int)pr.rows;
+    const int panel = pr.iterations == 32 ? 32 : 16;
     cudaStream_t s;
     RG_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     float* A = nullptr;
@@ -407,9 +409,9 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
         const char* key;
         int threads;
         lud::variant_info(vi, &g0, &fn, &key, &threads);
-        if (lud::kInternal[vi].p != 16) continue;
-        for (int bx : {1, 2, 4, 7, 8})
-            for (int by : {1, 2}) {
+        if (lud::kInternal[vi].p != panel) continue;
+        for (int bx : {1, 2, 4, 7})
+            for (int by : {1, 2, 4}) {
                 rodinia_tune_row row;
                 memset(&row, 0, sizeof row);
                 row.g = g0;
@@ -417,7 +419,7 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
                 row.g.block_y = by;
                 row.median_ms = -1.f;
                 lud::Plan pl;
-                rodinia_status cs = lud::plan(row.g, 16, &pl);
+                rodinia_status cs = lud::plan(row.g, panel, &pl);
                 const PtxasStats* ps = find_stats(key);
                 row.regs = ps ? ps->regs : -1;
                 row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
@@ -471,7 +473,7 @@ extern "C" rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const 
     rodinia_granularity gg;
     if (!gran_is_zero(g)) gg = *g;
     else {
-        rodinia_problem pb{n, n, 1, 1};
+        rodinia_problem pb{n, n, panel == 32 ? 32 : 16, 1};
         if (!tune_cache_lookup(RODINIA_LUD, pb, &gg)) gg = default_gran(RODINIA_LUD, pb);
     }
     lud::Plan pl;
