@@ -136,44 +136,86 @@ __device__ __forceinline__ void hs_ld(const float* __restrict__ base, int row, i
     }
 }
 
-// Loads are prefetched three rows ahead (register queues tq/pq, period 3 like the rings).  The
-// power row consumed by level 1 is parked in a per-warp shared-memory ring of H rows from which
-// levels 2..H read it back in later steps (each lane reads only its own columns, so no
-// synchronisation is needed); this replaces H-1 global re-loads per step.
-template <int V, int H, int K, bool EC, bool ER>
-__device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&tq)[3][V], float (&pq)[3][V],
-                                               float* __restrict__ psm, const float* __restrict__ tin,
-                                               const float* __restrict__ pw, float* __restrict__ tout,
-                                               int s, int g0, int R, int C, int ylo, int yhi, int sc0, int col0,
-                                               const HsCoef& cf) {
-    constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
-    // level 0 takes T row g0; level 1 takes P row g0-1; refill both queues three rows ahead
-    float p1[V];
+// Input rows stream through per-lane cp.async rings in shared memory (lane-private slots, so no
+// barrier): the T ring holds HS_DT rows, requested HS_DT-1 steps ahead; the P ring additionally
+// keeps each power row for the H steps during which levels 1..H read it (depth HsRing<H>::DP).
+// Rows outside [0, R) are zero-filled (their values only feed cells that are never stored).
+constexpr int HS_DT = 8;
+template <int H>
+struct HsRing {
+    static constexpr int need = HS_DT + H;
+    static constexpr int DP = need <= 8 ? 8 : (need <= 16 ? 16 : 32);
+};
+
+template <int V, bool EC>
+__device__ __forceinline__ void hs_issue_row(float* dst_base, const float* __restrict__ src_base, int row, int R,
+                                             int C, int col0, int sc0, int slot) {
+    float* dst = dst_base + slot * 32 * V + sc0;
+    const bool rok = row >= 0 && row < R;
+    const float* src = src_base + (size_t)(rok ? row : 0) * C;
+    if (!EC && V % 4 == 0) {
 #pragma unroll
-    for (int v = 0; v < V; ++v) { ring[0][S2][v] = tq[K][v]; p1[v] = pq[K][v]; }
-    hs_ld<V, EC, ER>(tin, g0 + 3, R, C, col0, tq[K]);
-    hs_ld<V, EC, ER>(pw, g0 + 2, R, C, col0, pq[K]);
-    const int sb = s % H;
-    if (H > 1) {
-        float* dst = psm + (sb * 32 * V) + sc0;
+        for (int q = 0; q < V / 4; ++q)
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + 4 * q)),
+                         "l"(src + col0 + 4 * q), "r"(rok ? 16 : 0));
+    } else if (!EC && V == 2) {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+                     "l"(src + col0), "r"(rok ? 8 : 0));
+    } else {
 #pragma unroll
-        for (int v = 0; v < V; ++v) dst[v] = p1[v];
+        for (int v = 0; v < V; ++v) {
+            const int c = col0 + v;
+            const bool ok = rok && c >= 0 && c < C;
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + v)),
+                         "l"(ok ? src + c : src_base), "r"(ok ? 4 : 0));
+        }
     }
+}
+
+template <int V>
+__device__ __forceinline__ void hs_read_row(const float* base, int sc0, int slot, float (&o)[V]) {
+    const float* p = base + slot * 32 * V + sc0;
+    if (V % 4 == 0) {
+#pragma unroll
+        for (int q = 0; q < V / 4; ++q) {
+            const float4 t = reinterpret_cast<const float4*>(p)[q];
+            o[(4 * q) % V] = t.x; o[(4 * q + 1) % V] = t.y; o[(4 * q + 2) % V] = t.z; o[(4 * q + 3) % V] = t.w;
+        }
+    } else {
+#pragma unroll
+        for (int v = 0; v < V; ++v) o[v] = p[v];
+    }
+}
+
+// Request the rows step `s` will consume: T row ystart+s into slot s % HS_DT, P row ystart+s-1
+// into slot s % DP (one commit group per step).
+template <int V, int H, bool EC>
+__device__ __forceinline__ void hs_issue_step(float* tring, float* pring, const float* __restrict__ tin,
+                                              const float* __restrict__ pw, int s, int ystart, int R, int C,
+                                              int col0, int sc0) {
+    hs_issue_row<V, EC>(tring, tin, ystart + s, R, C, col0, sc0, s & (HS_DT - 1));
+    hs_issue_row<V, EC>(pring, pw, ystart + s - 1, R, C, col0, sc0, s & (HsRing<H>::DP - 1));
+    asm volatile("cp.async.commit_group;\n" ::);
+}
+
+template <int V, int H, int K, bool EC, bool ER>
+__device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tring, float* pring,
+                                               const float* __restrict__ tin, const float* __restrict__ pw,
+                                               float* __restrict__ tout, int s, int ystart, int R, int C, int ylo,
+                                               int yhi, int sc0, int col0, const HsCoef& cf) {
+    constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
+    constexpr int DP = HsRing<H>::DP;
+    const int g0 = ystart + s;
+    // this step's rows have landed once at most HS_DT-2 later groups are pending
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(HS_DT - 2));
+    hs_read_row<V>(tring, sc0, s & (HS_DT - 1), ring[0][S2]);  // level 0 = T row g0
+    hs_issue_step<V, H, EC>(tring, pring, tin, pw, s + HS_DT - 1, ystart, R, C, col0, sc0);
 
 #pragma unroll
     for (int l = 0; l < H; ++l) {
-        const int g = g0 - l - 1;  // row computed by level l+1
+        const int g = g0 - l - 1;  // row computed by level l+1 (its power row was level 1's at step s-l)
         float pv[V];
-        if (l == 0) {
-#pragma unroll
-            for (int v = 0; v < V; ++v) pv[v] = p1[v];
-        } else {
-            int slot = sb + H - l;
-            slot -= (slot >= H) ? H : 0;
-            const float* src = psm + slot * 32 * V + sc0;
-#pragma unroll
-            for (int v = 0; v < V; ++v) pv[v] = src[v];
-        }
+        hs_read_row<V>(pring, sc0, (s - l) & (DP - 1), pv);
         const bool top = ER && (g == 0), bot = ER && (g == R - 1);
         const float wnb = __shfl_up_sync(0xffffffffu, ring[l][S1][V - 1], 1);
         const float enb = __shfl_down_sync(0xffffffffu, ring[l][S1][0], 1);
@@ -221,7 +263,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float (&t
 template <int V, int H, bool EC, bool ER>
 __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
                                                const float* __restrict__ pw,
-                                               float* __restrict__ tout, float* __restrict__ psm, int R,
+                                               float* __restrict__ tout, float* tring, float* pring, int R,
                                                int C, int y0, int y1, int sc0, int col0, const HsCoef& cf) {
     float ring[H][3][V];
 #pragma unroll
@@ -232,20 +274,17 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
             for (int v = 0; v < V; ++v) ring[l][k][v] = 0.0f;
     const int ystart = y0 - H;
     const int nsteps = (y1 - y0) + 2 * H;
-    float tq[3][V], pq[3][V];
 #pragma unroll
-    for (int k = 0; k < 3; ++k) {
-        hs_ld<V, EC, ER>(tin, ystart + k, R, C, col0, tq[k]);
-        hs_ld<V, EC, ER>(pw, ystart - 1 + k, R, C, col0, pq[k]);
-    }
+    for (int k = 0; k < HS_DT - 1; ++k) hs_issue_step<V, H, EC>(tring, pring, tin, pw, k, ystart, R, C, col0, sc0);
     int s = 0;
     for (; s + 3 <= nsteps; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s, ystart + s, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 1, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 1, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 2, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 2, ystart + s + 2, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 2, EC, ER>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf);
     }
-    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s, ystart + s, R, C, y0, y1, sc0, col0, cf);
-    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tq, pq, psm, tin, pw, tout, s + 1, ystart + s + 1, R, C, y0, y1, sc0, col0, cf);
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf);
+    asm volatile("cp.async.wait_group 0;\n" ::);  // drain before the rings are reused
 }
 
 // One warp per CTA: every branch condition derives from blockIdx and kernel arguments only, so
@@ -263,9 +302,10 @@ __global__ void __launch_bounds__(32, OCC)
     const int sc0 = (int)threadIdx.x * V;
     const int y0 = blockIdx.y * chunk;
     const int y1 = min(y0 + chunk, R);
-    // rows touched: T [y0-H, y1+H+2], P [y0-H-1, y1+H+1] (prefetch queues run 3 rows ahead)
-    const bool er = (y0 - H - 1 < 0) || (y1 + H + 2 > R - 1);
-    __shared__ __align__(16) float psm[H * 32 * V];
+    // rows computed: [y0-H, y1+H); ER selects the row-clamp path near the grid's top/bottom
+    const bool er = (y0 - H - 1 < 0) || (y1 + H > R - 1);
+    __shared__ __align__(16) float tring[HS_DT * 32 * V];
+    __shared__ __align__(16) float pring[HsRing<H>::DP * 32 * V];
     for (int bi = 0; bi < bands_per_cta; ++bi) {
         const int band = blockIdx.x * bands_per_cta + bi;
         if (band * OW >= C) return;
@@ -273,13 +313,13 @@ __global__ void __launch_bounds__(32, OCC)
         const int col0 = bstart + sc0;
         const bool ec = !vec_ok || bstart < 0 || bstart + SW > C;
         if (!ec && !er)
-            hs_stream_body<V, H, false, false>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, false, false>(tin, pw, tout, tring, pring, R, C, y0, y1, sc0, col0, cf);
         else if (ec && !er)
-            hs_stream_body<V, H, true, false>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, true, false>(tin, pw, tout, tring, pring, R, C, y0, y1, sc0, col0, cf);
         else if (!ec && er)
-            hs_stream_body<V, H, false, true>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, false, true>(tin, pw, tout, tring, pring, R, C, y0, y1, sc0, col0, cf);
         else
-            hs_stream_body<V, H, true, true>(tin, pw, tout, psm, R, C, y0, y1, sc0, col0, cf);
+            hs_stream_body<V, H, true, true>(tin, pw, tout, tring, pring, R, C, y0, y1, sc0, col0, cf);
     }
 }
 

@@ -93,10 +93,11 @@ rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
     switch (k) {
         case RODINIA_HOTSPOT:
             // B200 default (measured on 16384^2): streaming temporal blocking,
-            // 4 columns per lane, 4 steps per launch, 1 band per CTA, 64-row chunks.
-            if (p.iterations >= 4 && p.cols >= 128) return gran(4, 1, 1, 4, 4, 1, RODINIA_STREAM);
+            // 4 columns per lane, 8 steps per launch, 1 band per CTA, 128-row chunks,
+            // register budget for 12 CTAs/SM.
+            if (p.iterations >= 8 && p.cols >= 128) return gran(4, 1, 1, 8, 8, 1, RODINIA_STREAM | RODINIA_OCC(12));
             return gran(4, 1, 1, 1, 1, 1);
-        case RODINIA_SRAD: return gran(4, 1, 1, 1, 1, 1);
+        case RODINIA_SRAD: return gran(4, 1, 1, 2, 1, 1, RODINIA_STREAM);
         case RODINIA_PATHFINDER: return gran(4, 1, 1, 1, 8, 1);
         case RODINIA_LUD:  // measured on B200 at n = 8192
             return p.iterations == 32 ? gran(2, 4, 4, 2, 1, 1) : gran(4, 2, 2, 2, 1, 1);
