@@ -134,6 +134,115 @@ __global__ void __launch_bounds__(256)
 #endif
 }
 
+// ------------------------------------------------------------------ warp-band family
+// pf_band<CELLS> (flags RODINIA_STREAM): one warp per CTA owns a band of 32*CELLS contiguous
+// columns (CELLS contiguous ints per lane, 128-bit accesses) and runs all h rows of a launch
+// without any block barrier: row neighbours come from registers and two warp shuffles.  Wall
+// rows stream through a per-lane cp.async ring in shared memory PF_D-1 rows ahead.  The band's
+// halo is h rounded up to 4 columns per side (keeps 16-byte alignment).
+constexpr int PF_D = 8;
+
+template <int CELLS, bool EC>
+__device__ __forceinline__ void pf_issue(int32_t* ring, const int32_t* __restrict__ wall, int row, int C,
+                                         int col0, int lane, int slot) {
+    // layout [slot][q][lane][4]: for a fixed 16-byte chunk q the 32 lanes are contiguous, so the
+    // 128-bit shared stores and loads are bank-conflict free for any CELLS
+    int32_t* dst = ring + (slot * (CELLS / 4) * 32 + lane) * 4;
+    const int32_t* src = wall + (size_t)row * C;
+    if (!EC) {
+#pragma unroll
+        for (int q = 0; q < CELLS / 4; ++q)
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + q * 128)),
+                         "l"(src + col0 + 4 * q));
+    } else {
+#pragma unroll
+        for (int k = 0; k < CELLS; ++k) {
+            const int c = col0 + k;
+            const bool ok = c >= 0 && c < C;
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + (k / 4) * 128 + (k % 4))),
+                         "l"(ok ? src + c : wall), "r"(ok ? 4 : 0));
+        }
+    }
+    asm volatile("cp.async.commit_group;\n" ::);
+}
+
+template <int CELLS, bool EC>
+__device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, const int32_t* __restrict__ prev_in,
+                                             int32_t* __restrict__ next_out, int32_t* ring, int C, int r0, int h,
+                                             int b0, int band_out, int col0, int lane) {
+#pragma unroll
+    for (int i = 0; i < PF_D - 1; ++i)
+        if (i < h) pf_issue<CELLS, EC>(ring, wall, r0 + 1 + i, C, col0, lane, i);
+        else asm volatile("cp.async.commit_group;\n" ::);
+#if __CUDA_ARCH__ >= 900
+    cudaGridDependencySynchronize();  // PDL: prev_in is produced by the previous launch
+#endif
+    int32_t v[CELLS];
+    if (!EC) {
+#pragma unroll
+        for (int q = 0; q < CELLS / 4; ++q) {
+            const int4 t = *reinterpret_cast<const int4*>(prev_in + col0 + 4 * q);
+            v[4 * q] = t.x; v[(4 * q + 1) % CELLS] = t.y; v[(4 * q + 2) % CELLS] = t.z; v[(4 * q + 3) % CELLS] = t.w;
+        }
+    } else {
+#pragma unroll
+        for (int k = 0; k < CELLS; ++k) v[k] = (col0 + k >= 0 && col0 + k < C) ? prev_in[col0 + k] : 0;
+    }
+    for (int i = 0; i < h; ++i) {
+        asm volatile("cp.async.wait_group %0;\n" ::"n"(PF_D - 2));
+        int32_t w[CELLS];
+        const int32_t* src = ring + ((i & (PF_D - 1)) * (CELLS / 4) * 32 + lane) * 4;
+#pragma unroll
+        for (int q = 0; q < CELLS / 4; ++q) {
+            const int4 t = reinterpret_cast<const int4*>(src)[q * 32];
+            w[4 * q] = t.x; w[(4 * q + 1) % CELLS] = t.y; w[(4 * q + 2) % CELLS] = t.z; w[(4 * q + 3) % CELLS] = t.w;
+        }
+        if (i + PF_D - 1 < h) pf_issue<CELLS, EC>(ring, wall, r0 + i + PF_D, C, col0, lane, (i + PF_D - 1) & (PF_D - 1));
+        else asm volatile("cp.async.commit_group;\n" ::);
+        const int32_t lnb = __shfl_up_sync(0xffffffffu, v[CELLS - 1], 1);
+        const int32_t rnb = __shfl_down_sync(0xffffffffu, v[0], 1);
+        int32_t nv[CELLS];
+#pragma unroll
+        for (int k = 0; k < CELLS; ++k) {
+            int32_t l = k > 0 ? v[k > 0 ? k - 1 : 0] : lnb;
+            int32_t r = k < CELLS - 1 ? v[k < CELLS - 1 ? k + 1 : 0] : rnb;
+            if (EC) {
+                const int c = col0 + k;
+                if (c <= 0) l = v[k];
+                if (c >= C - 1) r = v[k];
+            }
+            nv[k] = w[k] + min(min(l, v[k]), r);
+        }
+#pragma unroll
+        for (int k = 0; k < CELLS; ++k) v[k] = nv[k];
+    }
+    asm volatile("cp.async.wait_group 0;\n" ::);
+#pragma unroll
+    for (int k = 0; k < CELLS; ++k) {
+        const int c = col0 + k;
+        if (c >= b0 && c < b0 + band_out && c < C) next_out[c] = v[k];
+    }
+#if __CUDA_ARCH__ >= 900
+    cudaTriggerProgrammaticLaunchCompletion();
+#endif
+}
+
+template <int CELLS>
+__global__ void __launch_bounds__(32)
+    pf_band(const int32_t* __restrict__ wall, const int32_t* __restrict__ prev_in, int32_t* __restrict__ next_out,
+            int R, int C, int r0, int h, int band_out) {
+    __shared__ __align__(16) int32_t ring[PF_D * 32 * CELLS];
+    const int lane = threadIdx.x;
+    const int halo = (h + 3) & ~3;
+    const int b0 = blockIdx.x * band_out;
+    const int s0 = b0 - halo;
+    const int col0 = s0 + lane * CELLS;
+    const bool ec = ((C & 3) != 0) || s0 < 0 || s0 + 32 * CELLS > C;
+    if (ec) pf_band_body<CELLS, true>(wall, prev_in, next_out, ring, C, r0, h, b0, band_out, col0, lane);
+    else pf_band_body<CELLS, false>(wall, prev_in, next_out, ring, C, r0, h, b0, band_out, col0, lane);
+    (void)R;
+}
+
 namespace pathfinder {
 
 typedef void (*PfFn)(const int32_t*, const int32_t*, int32_t*, int, int, int, int, int);
@@ -154,8 +263,15 @@ static const Variant* find(int cells, int mode) {
     return nullptr;
 }
 
+struct BandVariant { int cells; PfFn fn; const char* key; };
+static const BandVariant kBand[] = {
+    {4, pf_band<4>, "void rg::pf_band<4>"},   {8, pf_band<8>, "void rg::pf_band<8>"},
+    {16, pf_band<16>, "void rg::pf_band<16>"}, {32, pf_band<32>, "void rg::pf_band<32>"},
+};
+
 struct Plan {
     const Variant* v;
+    const BandVariant* band;  // warp-band family (flags & RODINIA_STREAM)
     int threads, h, band_out, launches;
 };
 
@@ -166,9 +282,27 @@ rodinia_status plan(const rodinia_granularity& g, int64_t R, int64_t C, Plan* p)
                                                    "thread_y = block_y = 1 (%s)", gran_str(g).c_str());
     if (g.index_mode != 0 && g.index_mode != 1)
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: index_mode must be 0 or 1");
-    if (g.flags & RODINIA_STREAM)
-        return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: no stream family");
     const int t = g.thread_x;
+    p->band = nullptr;
+    if (g.flags & RODINIA_STREAM) {
+        if (g.index_mode != 1 || (g.flags & RODINIA_FAITHFUL))
+            return set_error(RODINIA_E_NOT_BUILT, "pathfinder: the warp-band family is index_mode 1, non-faithful");
+        const int cells = t * g.block_x;
+        for (const auto& b : kBand)
+            if (b.cells == cells) p->band = &b;
+        if (!p->band) return set_error(RODINIA_E_NOT_BUILT, "pathfinder: warp-band with %d cells/lane not built", cells);
+        p->v = nullptr;
+        p->threads = 32;
+        const int64_t steps = R - 1;
+        p->h = (int)std::min<int64_t>(g.temporal, std::max<int64_t>(steps, 1));
+        const int halo = (p->h + 3) & ~3;
+        p->band_out = (32 * cells - 2 * halo) & ~3;
+        if (p->band_out < 4)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: pyramid height %d too large for a %d-column band",
+                             p->h, 32 * cells);
+        p->launches = steps > 0 ? (int)((steps + p->h - 1) / p->h) : 0;
+        return RODINIA_OK;
+    }
     if ((g.flags & RODINIA_FAITHFUL) && (256 % t != 0))
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: thread factor %d does not divide the "
                                                    "256-thread block (PAPER.md:237)", t);
@@ -197,8 +331,9 @@ rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R
         return RODINIA_OK;
     }
     const int nwarps = p.threads / 32;
-    const size_t smem = (size_t)2 * nwarps * 2 * p.v->cells * sizeof(int32_t);
+    const size_t smem = p.band ? 0 : (size_t)2 * nwarps * 2 * p.v->cells * sizeof(int32_t);
     const int grid = (C + p.band_out - 1) / p.band_out;
+    PfFn fn = p.band ? p.band->fn : p.v->fn;
     const int32_t* src = wall;  // row 0 of the wall is the initial cost
     int r0 = 0;
     for (int l = 0; l < p.launches; ++l) {
@@ -214,8 +349,7 @@ rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R
         attr[0].val.programmaticStreamSerializationAllowed = 1;
         cfg.attrs = attr;
         cfg.numAttrs = l > 0 ? 1 : 0;
-        RG_CUDA(cudaLaunchKernelEx(&cfg, p.v->fn, wall, (const int32_t*)src, dst, R, C, r0, h,
-                                   p.band_out));
+        RG_CUDA(cudaLaunchKernelEx(&cfg, fn, wall, (const int32_t*)src, dst, R, C, r0, h, p.band_out));
         count_launch();
         src = dst;
         r0 += h;
@@ -223,9 +357,18 @@ rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R
     return RODINIA_OK;
 }
 
-int num_variants() { return (int)(sizeof(kVariants) / sizeof(kVariants[0])); }
+int num_variants() { return (int)(sizeof(kVariants) / sizeof(kVariants[0]) + sizeof(kBand) / sizeof(kBand[0])); }
 
 void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    const int nv = (int)(sizeof(kVariants) / sizeof(kVariants[0]));
+    if (i >= nv) {
+        const auto& b = kBand[i - nv];
+        *g = gran(b.cells, 1, 1, 1, 99, 1, RODINIA_STREAM);
+        *fn = (const void*)b.fn;
+        *key = b.key;
+        *threads = 32;
+        return;
+    }
     const auto& v = kVariants[i];
     *g = gran(v.cells, 1, 1, 1, 20, v.mode);
     *fn = (const void*)v.fn;
@@ -292,7 +435,7 @@ rodinia_status tune_pathfinder(const rodinia_problem& pr, int reps, rodinia_gran
         for (int h : {4, 8, 12, 20, 33, 50, 99, 1 << 20}) {
             rodinia_tune_row row;
             memset(&row, 0, sizeof row);
-            row.g = gran(g0.thread_x, 1, 1, 1, h, g0.index_mode);
+            row.g = gran(g0.thread_x, 1, 1, 1, h, g0.index_mode, g0.flags);
             row.median_ms = -1.f;
             pathfinder::Plan p;
             rodinia_status cs = pathfinder::plan(row.g, R, C, &p);
@@ -300,7 +443,11 @@ rodinia_status tune_pathfinder(const rodinia_problem& pr, int reps, rodinia_gran
             row.regs = ps ? ps->regs : -1;
             row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
             row.threads = threads;
-            if (cs == RODINIA_OK) {
+            if (cs == RODINIA_OK && p.band) {
+                row.smem_bytes = PF_D * 32 * p.band->cells * 4;
+                row.ctas_per_sm = ctas_per_sm(fn, 32, 0);
+                cs = filter_decision(ps, 32, 0, 0);
+            } else if (cs == RODINIA_OK) {
                 row.smem_bytes = (int)((size_t)2 * (p.threads / 32) * 2 * p.v->cells * 4);
                 row.ctas_per_sm = ctas_per_sm(fn, p.threads, row.smem_bytes);
                 cs = filter_decision(ps, p.threads, row.smem_bytes, 0);

@@ -22,6 +22,13 @@ def timeit(g, batch=200):
     for _ in range(3):
         e0.record(); graph.replay(); e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1) / batch)
     return sorted(ts)[1]
+for cells in (4, 8, 16, 32):
+    for h in (16, 24, 33, 50, 99):
+        g = (cells, 1, 1, 1, h, 1, 2)
+        try:
+            res.append((timeit(g), g))
+        except Exception as e:
+            print(g, e)
 for t in range(1, 9):
     for b in (1, 2, 4):
         for h in (8, 16, 33, 50, 99):
