@@ -363,16 +363,47 @@ def run_ours(args):
             "kernel": "hs_stream" if g.flags & rg.RODINIA_STREAM else "hs_direct",
             "bytes_per_launch": bytes_per_launch, "avg_launch_ms": avg_launch_ms,
             "updates_per_launch": rows_local * N * h}
+    # The same kernel against the FP32 SIMT roof: hs_cell is 3 FADD + 6 FFMA =
+    # 15 flop per cell-update; peak = 148 SMs x 128 lanes x 2 flop x 1.965 GHz = 74.4 TFLOP/s.
+    # With H steps per launch the kernel sits near the ridge, so both fractions are reported.
+    fp32_peak = 148 * 128 * 2 * 1.965e9 / 1e12
+    ach_tf = 15.0 * rows_local * N * h / (avg_launch_ms * 1e-3) / 1e12
+    roof_alu = {"bound": "alu", "achieved": ach_tf, "peak": fp32_peak, "unit": "TFLOP/s",
+                "frac": ach_tf / fp32_peak, "flop_per_update": 15,
+                "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
 
     # ---- uncoarsened variant (same timed protocol, fewer steps)
     unc_ms = None
     if not args.no_extra:
         unc_ms = _max_over_ranks(_time_steps(lambda: step(UNC), 1, 1, stream), ws)
 
+    # ---- e2e at N > 1: each rank copies its slab from pinned host memory, solves through the
+    # row-slab API, copies its slab back; max over ranks
+    e2e_dist = None
+    if ws > 1:
+        th = torch.empty(t.shape, dtype=torch.float32, pin_memory=True)
+        ph = torch.empty(t.shape, dtype=torch.float32, pin_memory=True)
+        oh = torch.empty(t.shape, dtype=torch.float32, pin_memory=True)
+        th.copy_(t.cpu()); ph.copy_(p.cpu())
+        td, pd_, od = torch.empty_like(t), torch.empty_like(t), torch.empty_like(t)
+        def e2e_step():
+            td.copy_(th, non_blocking=True); pd_.copy_(ph, non_blocking=True)
+            comm.hotspot(td, pd_, od, N, iters, coeffs=coef, g=g, stream=stream)
+            oh.copy_(od, non_blocking=True)
+            torch.cuda.synchronize()
+        e2e_step()
+        _barrier(ws)
+        t0 = time.perf_counter()
+        e2e_step()
+        e2e_s = _max_over_ranks(time.perf_counter() - t0, ws)
+        e2e_dist = {"value": N * N * iters / e2e_s, "unit": "cell-updates/s",
+                    "h2d_bytes_per_step": 2 * 4 * N * N, "d2h_bytes_per_step": 4 * N * N,
+                    "ms_per_step": e2e_s * 1e3}
+
     result = None
     if rank == 0:
         # ---- e2e through the C ABI with pinned host buffers (1 GPU)
-        e2e = None
+        e2e = e2e_dist
         if ws == 1:
             th = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
             ph = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
@@ -420,6 +451,7 @@ def run_ours(args):
                        "l2": "no flush: working set 3 GiB >> 126 MB L2",
                        "tune_seconds": round(t_tune, 1)},
             "roofline": roof,
+            "roofline_alu": roof_alu,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches_timed,
