@@ -151,9 +151,10 @@ __device__ __forceinline__ void lud_tile_io(float* A, int n, int cx, int cy, flo
     }
 }
 
+// register budget: >= 512 resident threads per SM (<= 128 registers per thread)
 template <int P, int TX, int TY, int MODE>
 __global__ void __launch_bounds__((P / TX) * (P / TY),
-                                  (1024 / ((P / TX) * (P / TY))) < 32 ? (1024 / ((P / TX) * (P / TY))) : 32)
+                                  (512 / ((P / TX) * (P / TY))) < 32 ? ((512 / ((P / TX) * (P / TY))) > 0 ? (512 / ((P / TX) * (P / TY))) : 1) : 32)
     lud_internal(float* const* __restrict__ slot, int n, int k, int bx, int by) {
     float* A = *slot;
     extern __shared__ __align__(16) float lsm[];
@@ -167,15 +168,38 @@ __global__ void __launch_bounds__((P / TX) * (P / TY),
     const int tid = threadIdx.y * NTX + threadIdx.x;
     float av[TY][TX];
     lud_tile_io<P, TX, TY, MODE>(A, n, cx0, cy0, av, true);  // first tile's A, before staging
-    for (int e = tid; e < bx * P * P; e += NT) {
-        const int b = e / (P * P), rem = e - b * P * P, i = rem / P, c = rem - i * P;
-        const int gc = cx0 + b * P + c;
-        Ush[(b * P + i) * LD + c] = gc < n ? A[(size_t)(o + i) * n + gc] : 0.f;
+    // Stage U12 (row-major, 128-bit) and L21 (transposed) tiles.  Index math uses only the
+    // compile-time tile size; the per-tile loops are over the runtime block factors.
+    const bool vec = (n & 3) == 0;
+    for (int b = 0; b < bx; ++b) {
+        const int cb = cx0 + b * P;
+        for (int e4 = tid; e4 < P * P / 4; e4 += NT) {
+            const int i = e4 / (P / 4), c = 4 * (e4 % (P / 4));
+            float4 u = make_float4(0.f, 0.f, 0.f, 0.f);
+            const float* src = A + (size_t)(o + i) * n + cb + c;
+            if (vec && cb + c + 4 <= n) u = *reinterpret_cast<const float4*>(src);
+            else {
+                if (cb + c < n) u.x = src[0];
+                if (cb + c + 1 < n) u.y = src[1];
+                if (cb + c + 2 < n) u.z = src[2];
+                if (cb + c + 3 < n) u.w = src[3];
+            }
+            *reinterpret_cast<float4*>(Ush + (b * P + i) * LD + c) = u;
+        }
     }
-    for (int e = tid; e < by * P * P; e += NT) {
-        const int b = e / (P * P), rem = e - b * P * P, rr = rem / P, i = rem - rr * P;
-        const int gr = cy0 + b * P + rr;
-        Lsh[(b * P + i) * LD + rr] = gr < n ? A[(size_t)gr * n + o + i] : 0.f;
+    for (int b = 0; b < by; ++b) {
+        const int rb = cy0 + b * P;
+        for (int e4 = tid; e4 < P * P / 4; e4 += NT) {
+            const int rr = e4 / (P / 4), i = 4 * (e4 % (P / 4));
+            float4 l = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (rb + rr < n) {
+                const float* src = A + (size_t)(rb + rr) * n + o + i;
+                if (vec) l = *reinterpret_cast<const float4*>(src);
+                else l = make_float4(src[0], src[1], src[2], src[3]);
+            }
+            float* d = Lsh + (b * P + i) * LD + rr;
+            d[0] = l.x; d[LD] = l.y; d[2 * LD] = l.z; d[3 * LD] = l.w;
+        }
     }
     __syncthreads();
     const int ntiles = bx * by;
