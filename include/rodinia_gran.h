@@ -237,6 +237,13 @@ rodinia_status rodinia_srad_dist(rodinia_comm* comm, void* J_local, int64_t glob
                                  float lambda, int32_t niter, const rodinia_granularity* g,
                                  void* stream);
 
+/* Split a *total* coarsening factor over `ndims` (1..3) dimensions (footnote 4,
+ * "for a total factor of 16, we will coarsen the 3 dimensions with 4, 2, and 2
+ * respectively, whereas for 6 we will coarsen with 3, 2, and 1").  Reading G3: the prime factors
+ * of `total`, largest first, each go to the dimension with the smallest current factor (x wins
+ * ties).  Pure host call; out[0..2] receives the x, y, z factors (1 for unused dimensions). */
+rodinia_status rodinia_split_total(int32_t total, int32_t ndims, int32_t out[3]);
+
 /* ---------------------------------------------------------------------------------------
  * Misc. */
 const char* rodinia_last_error(void);

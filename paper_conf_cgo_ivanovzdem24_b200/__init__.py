@@ -120,6 +120,7 @@ _SIGS = {
     "rodinia_tune": ([_i32, ctypes.POINTER(Problem), _i32, _PG, ctypes.POINTER(TuneRow),
                       ctypes.POINTER(_i32)], _i32),
     "rodinia_resolve": ([_i32, ctypes.POINTER(Problem), _PG], _i32),
+    "rodinia_split_total": ([_i32, _i32, ctypes.POINTER(_i32)], _i32),
     "rodinia_slab": ([_i64, _i32, _i32, ctypes.POINTER(_i64), ctypes.POINTER(_i64)], _i32),
     "rodinia_comm_unique_id": ([ctypes.c_char_p], _i32),
     "rodinia_comm_init": ([ctypes.POINTER(_vp), _i32, _i32, ctypes.c_char_p], _i32),
@@ -322,6 +323,13 @@ def rodinia_resolve(kernel, rows: int, cols: int, iterations: int = 1, nranks: i
     g = Granularity()
     check(lib.rodinia_resolve(_kernel(kernel), ctypes.byref(p), ctypes.byref(g)), "rodinia_resolve")
     return g
+
+
+def rodinia_split_total(total: int, ndims: int = 3):
+    """Balance a total coarsening factor over ndims dimensions (footnote 4)."""
+    out = (_i32 * 3)()
+    check(lib.rodinia_split_total(int(total), int(ndims), out), "rodinia_split_total")
+    return tuple(out[:ndims])
 
 
 def rodinia_sync(stream=None):

@@ -323,3 +323,22 @@ extern "C" rodinia_status rodinia_resolve(rodinia_kernel k, const rodinia_proble
     *out = default_gran(k, *p);
     return RODINIA_OK;
 }
+
+extern "C" rodinia_status rodinia_split_total(int32_t total, int32_t ndims, int32_t out[3]) {
+    if (!out || total < 1 || ndims < 1 || ndims > 3) return set_error(RODINIA_E_INVALID, "split_total: bad arguments");
+    std::vector<int> primes;
+    int t = total;
+    for (int p = 2; (int64_t)p * p <= t; ++p)
+        while (t % p == 0) { primes.push_back(p); t /= p; }
+    if (t > 1) primes.push_back(t);
+    std::sort(primes.rbegin(), primes.rend());
+    int f[3] = {1, 1, 1};
+    for (int p : primes) {
+        int best = 0;
+        for (int d = 1; d < ndims; ++d)
+            if (f[d] < f[best]) best = d;
+        f[best] *= p;
+    }
+    for (int d = 0; d < 3; ++d) out[d] = f[d];
+    return RODINIA_OK;
+}

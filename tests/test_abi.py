@@ -105,3 +105,19 @@ def test_prune_rules():
     assert ptxas_filter.prune_reason(fat, 512, base_spill=0) == "occupancy"
     ok = ptxas_filter.KernelStats("w", "w", regs=40)
     assert ptxas_filter.prune_reason(ok, 256, base_spill=0) is None
+
+
+def test_split_total_footnote_examples():
+    # PAPER.md:189 (footnote 4): 16 -> (4, 2, 2), 6 -> (3, 2, 1)
+    assert rg.rodinia_split_total(16, 3) == (4, 2, 2)
+    assert rg.rodinia_split_total(6, 3) == (3, 2, 1)
+    # 2-D and edge cases of the reading (largest prime to the smallest current factor)
+    assert rg.rodinia_split_total(16, 2) == (4, 4)
+    assert rg.rodinia_split_total(14, 2) == (7, 2)
+    assert rg.rodinia_split_total(7, 3) == (7, 1, 1)
+    assert rg.rodinia_split_total(1, 3) == (1, 1, 1)
+    for t in range(1, 65):
+        x, y, z = rg.rodinia_split_total(t, 3)
+        assert x * y * z == t and max(x, y, z) <= t
+    with pytest.raises(rg.RodiniaError):
+        rg.rodinia_split_total(0, 3)
