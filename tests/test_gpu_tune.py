@@ -1,0 +1,85 @@
+"""Timing-driven tuning (TDO) and the compile-time filter on the GPU.
+
+The tuner times only variants that survive the ptxas filter, returns a
+legal granularity, stores it in the tune cache, and a later NULL-granularity call resolves to
+it; tuned results stay bitwise identical to the uncoarsened variant.
+"""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def rg():
+    import paper_conf_cgo_ivanovzdem24_b200 as m
+    return m
+
+
+def test_hotspot_tune_legal_and_cached(rg):
+    best, rows = rg.rodinia_tune("hotspot", 1024, 1024, 48, reps=1)
+    timed = [r for r in rows if r["status"] == 0 and r["median_ms"] > 0]
+    assert timed, rows[:3]
+    assert min(r["median_ms"] for r in timed) == pytest.approx(
+        [r["median_ms"] for r in timed if r["g"] == best.astuple()][0])
+    # every pruned row carries a filter / legality status, never a silent skip
+    assert all(r["status"] in (0, rg.RODINIA_E_FILTERED, rg.RODINIA_E_SMEM, rg.RODINIA_E_ILLEGAL_FACTOR,
+                               rg.RODINIA_E_NOT_BUILT) for r in rows)
+    assert all(r["spill_bytes"] == 0 for r in timed)  # new spills are never timed
+    assert rg.rodinia_resolve("hotspot", 1024, 1024, 48).astuple() == best.astuple()
+    T, P = synth.hotspot_inputs(1024, 1024)
+    t, p = torch.from_numpy(T).cuda(), torch.from_numpy(P).cuda()
+    c = rg.rodinia_hotspot_coeffs_rodinia(1024, 1024, 0.032, 0.032)
+    a = rg.rodinia_hotspot(t, p, 48, coeffs=c, g=None)          # resolves to the tuned variant
+    b = rg.rodinia_hotspot(t, p, 48, coeffs=c, g=rg.UNCOARSENED)
+    assert torch.equal(a, b)
+
+
+def test_srad_and_lud_tune(rg):
+    best, rows = rg.rodinia_tune("srad", 512, 512, 10, reps=1)
+    assert any(r["status"] == 0 for r in rows)
+    J = torch.from_numpy(synth.srad_input(512, 512)).cuda()
+    J2 = J.clone()
+    rg.rodinia_srad(J, 0, 127, 0, 127, 0.5, 10, g=best)
+    rg.rodinia_srad(J2, 0, 127, 0, 127, 0.5, 10, g=rg.UNCOARSENED)
+    assert torch.equal(J, J2)
+    for panel in (16, 32):
+        best, rows = rg.rodinia_tune("lud", 512, 512, panel, reps=1)
+        assert any(r["status"] == 0 for r in rows)
+        A = torch.from_numpy(synth.lud_rodinia_matrix(512)).cuda()
+        rg.rodinia_lud(A, panel, g=best)
+        assert torch.isfinite(A).all()
+
+
+def test_tune_cache_persists_across_processes(tmp_path):
+    cache = tmp_path / "tune.jsonl"
+    env = dict(os.environ, RODINIA_TUNE_CACHE=str(cache))
+    code1 = ("import sys; sys.path.insert(0, %r); import paper_conf_cgo_ivanovzdem24_b200 as rg, json;"
+             "b, _ = rg.rodinia_tune('pathfinder', 50, 20000, 1, reps=1); print(json.dumps(b.astuple()))" % ROOT)
+    code2 = ("import sys; sys.path.insert(0, %r); import paper_conf_cgo_ivanovzdem24_b200 as rg, json;"
+             "print(json.dumps(rg.rodinia_resolve('pathfinder', 50, 20000, 1).astuple()))" % ROOT)
+    out1 = subprocess.run([sys.executable, "-c", code1], env=env, capture_output=True, text=True, check=True)
+    out2 = subprocess.run([sys.executable, "-c", code2], env=env, capture_output=True, text=True, check=True)
+    assert json.loads(out1.stdout.strip().splitlines()[-1]) == json.loads(out2.stdout.strip().splitlines()[-1])
+    assert cache.exists() and cache.read_text().count("\n") >= 1
+
+
+def test_variant_tables_agree_with_runtime(rg):
+    # ptxas registers (compile-time table) vs the runtime's occupancy query: every kept variant
+    # fits at least one CTA per SM; every variant with new spills is pruned
+    for k in ("hotspot", "srad", "pathfinder", "lud"):
+        rows = rg.rodinia_variants(k)
+        assert rows, k
+        for r in rows:
+            if r["status"] == 0:
+                assert r["ctas_per_sm"] >= 1 and r["spill_bytes"] == 0, (k, r)
