@@ -138,9 +138,11 @@ __global__ void __launch_bounds__(256)
 // pf_band<CELLS> (flags RODINIA_STREAM): one warp per CTA owns a band of 32*CELLS contiguous
 // columns (CELLS contiguous ints per lane, 128-bit accesses) and runs all h rows of a launch
 // without any block barrier: row neighbours come from registers and two warp shuffles.  Wall
-// rows stream through a per-lane cp.async ring in shared memory PF_D-1 rows ahead.  The band's
+// rows stream through a per-lane cp.async ring in shared memory PfRing::D-1 rows ahead.  The band's
 // halo is h rounded up to 4 columns per side (keeps 16-byte alignment).
-constexpr int PF_D = 8;
+// ring depth (rows in flight); deeper rings (16-32) were measured slower (longer prologue)
+template <int CELLS>
+struct PfRing { static constexpr int D = 8; };
 
 template <int CELLS, bool EC>
 __device__ __forceinline__ void pf_issue(int32_t* ring, const int32_t* __restrict__ wall, int row, int C,
@@ -171,7 +173,7 @@ __device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, c
                                              int32_t* __restrict__ next_out, int32_t* ring, int C, int r0, int h,
                                              int b0, int band_out, int col0, int lane) {
 #pragma unroll
-    for (int i = 0; i < PF_D - 1; ++i)
+    for (int i = 0; i < PfRing<CELLS>::D - 1; ++i)
         if (i < h) pf_issue<CELLS, EC>(ring, wall, r0 + 1 + i, C, col0, lane, i);
         else asm volatile("cp.async.commit_group;\n" ::);
 #if __CUDA_ARCH__ >= 900
@@ -189,15 +191,15 @@ __device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, c
         for (int k = 0; k < CELLS; ++k) v[k] = (col0 + k >= 0 && col0 + k < C) ? prev_in[col0 + k] : 0;
     }
     for (int i = 0; i < h; ++i) {
-        asm volatile("cp.async.wait_group %0;\n" ::"n"(PF_D - 2));
+        asm volatile("cp.async.wait_group %0;\n" ::"n"(PfRing<CELLS>::D - 2));
         int32_t w[CELLS];
-        const int32_t* src = ring + ((i & (PF_D - 1)) * (CELLS / 4) * 32 + lane) * 4;
+        const int32_t* src = ring + ((i & (PfRing<CELLS>::D - 1)) * (CELLS / 4) * 32 + lane) * 4;
 #pragma unroll
         for (int q = 0; q < CELLS / 4; ++q) {
             const int4 t = reinterpret_cast<const int4*>(src)[q * 32];
             w[4 * q] = t.x; w[(4 * q + 1) % CELLS] = t.y; w[(4 * q + 2) % CELLS] = t.z; w[(4 * q + 3) % CELLS] = t.w;
         }
-        if (i + PF_D - 1 < h) pf_issue<CELLS, EC>(ring, wall, r0 + i + PF_D, C, col0, lane, (i + PF_D - 1) & (PF_D - 1));
+        if (i + PfRing<CELLS>::D - 1 < h) pf_issue<CELLS, EC>(ring, wall, r0 + i + PfRing<CELLS>::D, C, col0, lane, (i + PfRing<CELLS>::D - 1) & (PfRing<CELLS>::D - 1));
         else asm volatile("cp.async.commit_group;\n" ::);
         const int32_t lnb = __shfl_up_sync(0xffffffffu, v[CELLS - 1], 1);
         const int32_t rnb = __shfl_down_sync(0xffffffffu, v[0], 1);
@@ -231,7 +233,7 @@ template <int CELLS>
 __global__ void __launch_bounds__(32)
     pf_band(const int32_t* __restrict__ wall, const int32_t* __restrict__ prev_in, int32_t* __restrict__ next_out,
             int R, int C, int r0, int h, int band_out) {
-    __shared__ __align__(16) int32_t ring[PF_D * 32 * CELLS];
+    __shared__ __align__(16) int32_t ring[PfRing<CELLS>::D * 32 * CELLS];
     const int lane = threadIdx.x;
     const int halo = (h + 3) & ~3;
     const int b0 = blockIdx.x * band_out;
@@ -444,7 +446,7 @@ rodinia_status tune_pathfinder(const rodinia_problem& pr, int reps, rodinia_gran
             row.spill_bytes = ps ? ps->spill_stores + ps->spill_loads : -1;
             row.threads = threads;
             if (cs == RODINIA_OK && p.band) {
-                row.smem_bytes = PF_D * 32 * p.band->cells * 4;
+                row.smem_bytes = 8 * 32 * p.band->cells * 4;
                 row.ctas_per_sm = ctas_per_sm(fn, 32, 0);
                 cs = filter_decision(ps, 32, 0, 0);
             } else if (cs == RODINIA_OK) {
