@@ -190,6 +190,43 @@ def _time_steps(fn, steps, warmup, stream):
     return e0.elapsed_time(e1) / steps
 
 
+def _cpu_srad(n):
+    """fp64 C oracle on a 512-row sample of the n x n image, 20 iterations (cell-updates/s)."""
+    import oracle
+    import synth
+    J = synth.srad_input(512, n)
+    t0 = time.perf_counter()
+    oracle.srad(J, 0, 127, 0, 127, 0.5, 20)
+    dt = time.perf_counter() - t0
+    return {"value": 512 * n * 20 / dt, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
+            "sample": f"512x{n} rows x cols, 20 iterations ({dt:.1f} s), fp64 plain C"}
+
+
+def _cpu_pathfinder():
+    import oracle
+    import synth
+    w = synth.pathfinder_wall(100, 100000)
+    reps, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < 2.0:
+        oracle.pathfinder(w)
+        reps += 1
+    dt = (time.perf_counter() - t0) / reps
+    return {"value": 99 * 100000 / dt, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
+            "sample": f"full 100x100000 problem, {reps} calls, {dt*1e3:.2f} ms/call, int32 plain C"}
+
+
+def _cpu_lud():
+    import oracle
+    import synth
+    n = 1024
+    A = synth.lud_rodinia_matrix(n)
+    t0 = time.perf_counter()
+    oracle.lud(A)
+    dt = time.perf_counter() - t0
+    return {"value": (2 * n ** 3 / 3) / dt / 1e9, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"n={n} Rodinia matrix ({dt:.1f} s), fp64 plain C Doolittle"}
+
+
 def extra_workloads(rg, torch, tune: bool):
     """srad / pathfinder / lud at their BASELINE configs (1 GPU): tuned vs uncoarsened."""
     out = {}
@@ -224,6 +261,12 @@ def extra_workloads(rg, torch, tune: bool):
             res[name] = {"ms": ms, "cell_updates_per_s": n * n * it / (ms * 1e-3),
                          "g": list(g.astuple()) if hasattr(g, "astuple") else (list(g) if g else None)}
         res["speedup"] = res["uncoarsened"]["ms"] / res["tuned"]["ms"]
+        # roofline: 8 B per cell-update (J in, J out) at one iteration per launch
+        hbm, src = _peaks()
+        ach = 8.0 * res["tuned"]["cell_updates_per_s"] / 1e9
+        res["roofline"] = {"bound": "hbm", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm,
+                           "bytes_per_update": 8, "peak_source": src}
+        res["cpu_baseline"] = _cpu_srad(n)
         out["srad"] = res
     except Exception as e:  # noqa: BLE001
         out["srad"] = {"error": str(e)[:200]}
@@ -253,6 +296,13 @@ def extra_workloads(rg, torch, tune: bool):
             res[name] = {"ms_per_call": ms, "cell_updates_per_s": 99 * 100000 / (ms * 1e-3),
                          "g": list(g.astuple()) if hasattr(g, "astuple") else list(g)}
         res["speedup"] = res["uncoarsened"]["ms_per_call"] / res["tuned"]["ms_per_call"]
+        # 4 B of wall per cell-update; the DP is latency-bound (99 dependent rows)
+        hbm, src = _peaks()
+        ach = 4.0 * res["tuned"]["cell_updates_per_s"] / 1e9
+        res["roofline"] = {"bound": "latency", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm,
+                           "bytes_per_update": 4, "peak_source": src,
+                           "note": "wall is L2-resident across calls; time is the 99-row dependency chain"}
+        res["cpu_baseline"] = _cpu_pathfinder()
         out["pathfinder"] = res
     except Exception as e:  # noqa: BLE001
         out["pathfinder"] = {"error": str(e)[:200]}
@@ -272,6 +322,13 @@ def extra_workloads(rg, torch, tune: bool):
                          "g": list(g.astuple()) if hasattr(g, "astuple") else (list(g) if g else None)}
         res["speedup"] = res["uncoarsened"]["ms"] / res["tuned"]["ms"]
         res["speedup_panel32"] = res["uncoarsened"]["ms"] / res["tuned_panel32"]["ms"]
+        # FP32 SIMT roof: 2n^3/3 flop (tensor cores unused: TF32 would break the 1e-5 bar)
+        peak = 148 * 128 * 2 * 1.965e9 / 1e12
+        for key in ("tuned", "tuned_panel32"):
+            res[key]["roofline"] = {"bound": "alu", "achieved": res[key]["gflops"] / 1e3, "peak": peak,
+                                    "unit": "TFLOP/s", "frac": res[key]["gflops"] / 1e3 / peak,
+                                    "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
+        res["cpu_baseline"] = _cpu_lud()
         out["lud"] = res
     except Exception as e:  # noqa: BLE001
         out["lud"] = {"error": str(e)[:200]}
