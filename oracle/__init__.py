@@ -61,9 +61,10 @@ def _load():
             lib.oracle_srad.argtypes = [pd, l, l, l, l, l, l, d, i, pd]
             lib.oracle_pathfinder.argtypes = [pi32, l, l, pi32]
             lib.oracle_lud.argtypes = [pd, l]
+            lib.oracle_srad_v1.argtypes = [pd, l, l, d, i]
             for f in ("oracle_hotspot_coeffs_rodinia", "oracle_hotspot", "oracle_srad_q0sqr",
                       "oracle_srad_coeff", "oracle_srad_step", "oracle_srad",
-                      "oracle_pathfinder", "oracle_lud"):
+                      "oracle_pathfinder", "oracle_lud", "oracle_srad_v1"):
                 getattr(lib, f).restype = ctypes.c_int
             _lib = lib
     return _lib
@@ -141,6 +142,15 @@ def srad(J, r1, r2, c1, c2, lam: float, niter: int, return_q0: bool = False):
     q0 = np.zeros(max(niter, 1), dtype=np.float64)
     _chk(_load().oracle_srad(_p(J), R, C, r1, r2, c1, c2, float(lam), int(niter), _p(q0)), "srad")
     return (J, q0[:niter]) if return_q0 else J
+
+
+def srad_v1(image, lam: float, niter: int):
+    """Rodinia srad_v1: extract (exp(x/255)), niter iterations with whole-image statistics,
+    compress (log(J)*255); fp64."""
+    a = _f64(image).copy()
+    R, C = a.shape
+    _chk(_load().oracle_srad_v1(_p(a), R, C, float(lam), int(niter)), "srad_v1")
+    return a
 
 
 # --------------------------------------------------------------------------- pathfinder

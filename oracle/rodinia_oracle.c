@@ -267,3 +267,20 @@ int oracle_lud(double* a, long n) {
     }
     return ORACLE_OK;
 }
+
+/* ------------------------------------------------------------------------------------ */
+/* srad_v1 (Rodinia srad_v1 `extract`, `prepare`+`reduce`, `srad`, `srad2`, `compress`;
+ * DESIGN.md readings V1-V4).  The image (pixel values 0..255) is mapped to J = exp(image/255)
+ * (extract), niter srad iterations run with the statistics taken over the WHOLE image
+ * (srad_v1's ROI is rows 0..R-1, cols 0..C-1), and the result is mapped back with
+ * image = log(J)*255 (compress).  The per-iteration arithmetic is srad_v2's (pass 1, pass 2
+ * above).  image (R*C) is updated in place. */
+int oracle_srad_v1(double* image, long R, long C, double lambda, int niter) {
+    if (!image || R < 1 || C < 1 || niter < 0 || !isfinite(lambda)) return ORACLE_EINVAL;
+    size_t n = (size_t)R * (size_t)C;
+    for (size_t i = 0; i < n; ++i) image[i] = exp(image[i] / 255.0);
+    int st = oracle_srad(image, R, C, 0, R - 1, 0, C - 1, lambda, niter, NULL);
+    if (st) return st;
+    for (size_t i = 0; i < n; ++i) image[i] = log(image[i]) * 255.0;
+    return ORACLE_OK;
+}

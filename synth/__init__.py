@@ -16,6 +16,7 @@ import numpy as np
 __all__ = [
     "hotspot_inputs",
     "srad_input",
+    "srad_v1_image",
     "pathfinder_wall",
     "lud_rodinia_matrix",
     "lud_diag_dominant",
@@ -42,6 +43,19 @@ def hotspot_inputs(rows: int, cols: int, seed_t: int = 1, seed_p: int = 2):
 def srad_input(rows: int, cols: int, seed: int = 7):
     """srad_v2 image J0 = exp(U[0,1)) in [1, e) (Rodinia srad_v2 draws exp(rand()/RAND_MAX))."""
     return np.exp(_rng(seed).random((rows, cols))).astype(np.float32)
+
+
+def srad_v1_image(rows: int, cols: int, seed: int = 13):
+    """Synthetic ultrasound-like image for srad_v1 (Rodinia reads a 502x458 PGM; no dataset here):
+    a smooth intensity field (sum of low-frequency cosines) times Rayleigh speckle, clipped and
+    quantised to integer pixel values 0..255, returned as float32 (rows, cols)."""
+    rng = _rng(seed)
+    y = np.linspace(0.0, 1.0, rows)[:, None]
+    x = np.linspace(0.0, 1.0, cols)[None, :]
+    base = 0.55 + 0.25 * np.cos(3.1 * x + 0.7) * np.cos(2.3 * y) + 0.15 * np.cos(7.0 * (x + y))
+    speckle = rng.rayleigh(scale=0.8, size=(rows, cols))
+    img = np.clip(255.0 * base * speckle / 1.25, 0.0, 255.0)
+    return np.rint(img).astype(np.float32)
 
 
 def pathfinder_wall(rows: int, cols: int, seed: int = 9):

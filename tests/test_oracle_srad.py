@@ -144,3 +144,36 @@ def test_dependency_cone_outside_unchanged():
     mask[max(r1 - 2 * t, 0):r2 + t + 1, max(c1 - 2 * t, 0):c2 + t + 1] = True
     assert np.array_equal(out[~mask], J[~mask])
     assert not np.array_equal(out[mask], J[mask])
+
+
+# ----------------------------------------------------------------------------- srad_v1
+def test_srad_v1_is_extract_v2_whole_roi_compress():
+    # Rodinia srad_v1 = extract (exp(x/255)) + srad_v2 iterations with ROI = whole image +
+    # compress (log(J)*255) -- composition of independently pinned pieces
+    import synth
+    img = synth.srad_v1_image(37, 29)
+    J = np.exp(img.astype(np.float64) / 255.0)
+    ref = np.log(oracle.srad(J, 0, 36, 0, 28, 0.5, 6)) * 255.0
+    np.testing.assert_allclose(oracle.srad_v1(img, 0.5, 6), ref, rtol=0, atol=1e-10)
+
+
+def test_srad_v1_fixed_points():
+    import synth
+    img = synth.srad_v1_image(30, 40)
+    # lambda = 0 and niter = 0: only the exp/log round trip
+    np.testing.assert_allclose(oracle.srad_v1(img, 0.0, 5), img, rtol=0, atol=1e-9)
+    np.testing.assert_allclose(oracle.srad_v1(img, 0.5, 0), img, rtol=0, atol=1e-9)
+    flat = np.full((16, 20), 97.0)
+    np.testing.assert_allclose(oracle.srad_v1(flat, 0.5, 10), flat, rtol=0, atol=1e-9)
+
+
+def test_srad_v1_smooths_speckle():
+    # anisotropic diffusion reduces the coefficient of variation of a speckled image
+    import synth
+    img = synth.srad_v1_image(64, 64)
+    out = oracle.srad_v1(img, 0.5, 30)
+    def cv(a):
+        J = np.exp(a / 255.0)
+        return J.std() / J.mean()
+    assert cv(out) < 0.8 * cv(img)
+    assert out.min() >= img.min() - 1e-9 and out.max() <= img.max() + 1e-9  # maximum principle
