@@ -145,6 +145,16 @@ rodinia_status rodinia_srad_host(float* J, int64_t rows, int64_t cols, int64_t r
                                  int64_t c1, int64_t c2, float lambda, int32_t niter,
                                  const rodinia_granularity* g, void* stream);
 
+/* srad_v1 -- Rodinia srad_v1, the srad variant the paper evaluates, DESIGN.md
+ * readings V1-V4: extract J = exp(image/255); niter iterations of the srad arithmetic above with
+ * the statistics over the WHOLE image (srad_v1's ROI); compress image = log(J)*255.  image
+ * (rows x cols, pixel values in [0, 255], row-major) is updated in place.  Same granularity space
+ * as rodinia_srad. */
+rodinia_status rodinia_srad_v1(float* image, int64_t rows, int64_t cols, float lambda,
+                               int32_t niter, const rodinia_granularity* g, void* stream);
+rodinia_status rodinia_srad_v1_host(float* image, int64_t rows, int64_t cols, float lambda,
+                                    int32_t niter, const rodinia_granularity* g, void* stream);
+
 /* ---------------------------------------------------------------------------------------
  * pathfinder -- Rodinia pathfinder `dynproc_kernel` (min-cost path DP), P1-P6.
  *   prev = wall[0]; next[j] = wall[r][j] + min(prev[j-1], prev[j], prev[j+1]) (existing

@@ -112,6 +112,8 @@ _SIGS = {
     "rodinia_hotspot_host": ([_vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
     "rodinia_srad": ([_vp, _i64, _i64, _i64, _i64, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
     "rodinia_srad_host": ([_vp, _i64, _i64, _i64, _i64, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
+    "rodinia_srad_v1": ([_vp, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
+    "rodinia_srad_v1_host": ([_vp, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
     "rodinia_pathfinder": ([_vp, _i64, _i64, _vp, _PG, _vp], _i32),
     "rodinia_pathfinder_host": ([_vp, _i64, _i64, _vp, _PG, _vp], _i32),
     "rodinia_lud": ([_vp, _i64, _i32, _PG, _vp], _i32),
@@ -249,6 +251,24 @@ def rodinia_srad_host(J, r1, r2, c1, c2, lam: float, niter: int, g=None, stream=
     R, C = a.shape
     check(lib.rodinia_srad_host(ctypes.c_void_p(a.ctypes.data), R, C, r1, r2, c1, c2, float(lam),
                                 int(niter), _g(g), _stream(stream)), "rodinia_srad_host")
+    return a
+
+
+def rodinia_srad_v1(image, lam: float, niter: int, g=None, stream=None):
+    """Rodinia srad_v1 on image (R x C float32 CUDA tensor, pixel values 0..255, in place)."""
+    import torch
+    R, C = image.shape
+    check(lib.rodinia_srad_v1(_dev(image, torch.float32, "image"), R, C, float(lam), int(niter), _g(g),
+                              _stream(stream)), "rodinia_srad_v1")
+    return image
+
+
+def rodinia_srad_v1_host(image, lam: float, niter: int, g=None, stream=None):
+    import numpy as np
+    a = np.ascontiguousarray(image, dtype=np.float32).copy()
+    R, C = a.shape
+    check(lib.rodinia_srad_v1_host(ctypes.c_void_p(a.ctypes.data), R, C, float(lam), int(niter), _g(g),
+                                   _stream(stream)), "rodinia_srad_v1_host")
     return a
 
 
