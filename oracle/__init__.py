@@ -179,3 +179,37 @@ def lud_unpack(packed: np.ndarray):
     L = np.tril(packed, -1) + np.eye(n, dtype=packed.dtype)
     U = np.triu(packed)
     return L, U
+
+
+# --------------------------------------------------------------------------- hotspot3D
+def hotspot3d_coeffs(nx: int, ny: int, nz: int, chip_w: float = 0.016, chip_h: float = 0.016,
+                     t_chip: float = 0.0005):
+    """Rodinia hotspot3D constants -> dict(cc, cw, ce, cs, cn, cb, ct, sdc, amb), fp64."""
+    lib = _load()
+    lib.oracle_hotspot3d_coeffs.argtypes = [ctypes.c_long] * 3 + [ctypes.c_double] * 3 + [
+        ctypes.POINTER(ctypes.c_double)]
+    lib.oracle_hotspot3d_coeffs.restype = ctypes.c_int
+    out = np.zeros(9, dtype=np.float64)
+    _chk(lib.oracle_hotspot3d_coeffs(nx, ny, nz, chip_w, chip_h, t_chip, _p(out)), "hotspot3d_coeffs")
+    return dict(zip(("cc", "cw", "ce", "cs", "cn", "cb", "ct", "sdc", "amb"), out.tolist()))
+
+
+HS3D_KEYS = ("cc", "cw", "ce", "cs", "cn", "cb", "ct", "sdc", "amb")
+
+
+def hotspot3d(t0, power, iterations: int, coef: dict) -> np.ndarray:
+    """`iterations` Jacobi steps of Rodinia hotspot3D (7-point, clamped), fp64.  Arrays are
+    (nz, ny, nx), x fastest."""
+    lib = _load()
+    pd = ctypes.POINTER(ctypes.c_double)
+    lib.oracle_hotspot3d.argtypes = [pd, pd, pd, ctypes.c_long, ctypes.c_long, ctypes.c_long, ctypes.c_int, pd]
+    lib.oracle_hotspot3d.restype = ctypes.c_int
+    t0 = _f64(t0)
+    p = _f64(power)
+    if t0.ndim != 3 or p.shape != t0.shape:
+        raise ValueError("t0 and power must be equal-shaped (nz, ny, nx) arrays")
+    nz, ny, nx = t0.shape
+    cf = np.array([coef[k] for k in HS3D_KEYS], dtype=np.float64)
+    out = np.empty_like(t0)
+    _chk(lib.oracle_hotspot3d(_p(t0), _p(p), _p(out), nx, ny, nz, int(iterations), _p(cf)), "hotspot3d")
+    return out

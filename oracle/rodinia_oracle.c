@@ -284,3 +284,67 @@ int oracle_srad_v1(double* image, long R, long C, double lambda, int niter) {
     for (size_t i = 0; i < n; ++i) image[i] = log(image[i]) * 255.0;
     return ORACLE_OK;
 }
+
+/* ------------------------------------------------------------------------------------ */
+/* hotspot3D (Rodinia hotspot3D `hotspotOpt1` / `computeTempCPU`; readings T1-T4).
+ * Grid nx (x, fastest) x ny x nz, index c = z*nx*ny + y*nx + x.
+ * Chip constants as hotspot; cell sizes dx = chip_h/ny ... Rodinia: dx = chip_height/numRows,
+ * dy = chip_width/numCols, dz = t_chip/layers:
+ *   Cap = FACTOR_CHIP*SPEC_HEAT_SI*t_chip*dx*dy; Rx = dy/(2 K_SI t_chip dx);
+ *   Ry = dx/(2 K_SI t_chip dy); Rz = dz/(K_SI dx dy); dt = PRECISION / (MAX_PD/(FACTOR_CHIP t_chip SPEC_HEAT_SI))
+ *   sdc = dt/Cap; ce = cw = sdc/Rx; cn = cs = sdc/Ry; ct = cb = sdc/Rz; cc = 1 - (2ce + 2cn + 3ct)
+ * out[0..8] = {cc, cw, ce, cs, cn, cb, ct, sdc, amb}. */
+int oracle_hotspot3d_coeffs(long nx, long ny, long nz, double chip_w, double chip_h, double t_chip,
+                            double out[9]) {
+    if (nx < 1 || ny < 1 || nz < 1 || !(chip_w > 0) || !(chip_h > 0) || !(t_chip > 0) || !out)
+        return ORACLE_EINVAL;
+    const double k_si = 100.0, spec_heat_si = 1.75e6, factor_chip = 0.5, max_pd = 3.0e6;
+    const double precision = 0.001, amb = 80.0;
+    double dx = chip_h / (double)ny, dy = chip_w / (double)nx, dz = t_chip / (double)nz;
+    double cap = factor_chip * spec_heat_si * t_chip * dx * dy;
+    double rx = dy / (2.0 * k_si * t_chip * dx);
+    double ry = dx / (2.0 * k_si * t_chip * dy);
+    double rz = dz / (k_si * dx * dy);
+    double max_slope = max_pd / (factor_chip * t_chip * spec_heat_si);
+    double dt = precision / max_slope;
+    double sdc = dt / cap;
+    double ce = sdc / rx, cn = sdc / ry, ct = sdc / rz;
+    out[0] = 1.0 - (2.0 * ce + 2.0 * cn + 3.0 * ct);
+    out[1] = ce; out[2] = ce;   /* cw, ce */
+    out[3] = cn; out[4] = cn;   /* cs, cn */
+    out[5] = ct; out[6] = ct;   /* cb, ct */
+    out[7] = sdc;
+    out[8] = amb;
+    return ORACLE_OK;
+}
+
+/* `iters` Jacobi steps of the 7-point stencil, neighbours clamped to the grid:
+ *   T' = cc*c + cw*W + ce*E + cs*S + cn*N + cb*B + ct*T + sdc*P + ct*amb
+ * (W/E: x-1/x+1, N/S: y-1/y+1, B/T: z-1/z+1), summed left to right. */
+int oracle_hotspot3d(const double* t0, const double* p, double* out, long nx, long ny, long nz,
+                     int iters, const double cf[9]) {
+    if (!t0 || !p || !out || !cf || nx < 1 || ny < 1 || nz < 1 || iters < 0) return ORACLE_EINVAL;
+    const double cc = cf[0], cw = cf[1], ce = cf[2], cs = cf[3], cn = cf[4], cb = cf[5], ct = cf[6];
+    const double sdc = cf[7], amb = cf[8];
+    size_t n = (size_t)nx * ny * nz, plane = (size_t)nx * ny;
+    double* cur = (double*)malloc(n * sizeof(double));
+    double* nxt = (double*)malloc(n * sizeof(double));
+    if (!cur || !nxt) { free(cur); free(nxt); return ORACLE_ENOMEM; }
+    memcpy(cur, t0, n * sizeof(double));
+    for (int it = 0; it < iters; ++it) {
+        for (long z = 0; z < nz; ++z)
+            for (long y = 0; y < ny; ++y)
+                for (long x = 0; x < nx; ++x) {
+                    size_t c = (size_t)z * plane + (size_t)y * nx + x;
+                    size_t w = x == 0 ? c : c - 1, e = x == nx - 1 ? c : c + 1;
+                    size_t nn = y == 0 ? c : c - nx, s = y == ny - 1 ? c : c + nx;
+                    size_t b = z == 0 ? c : c - plane, t = z == nz - 1 ? c : c + plane;
+                    nxt[c] = cc * cur[c] + cw * cur[w] + ce * cur[e] + cs * cur[s] + cn * cur[nn] +
+                             cb * cur[b] + ct * cur[t] + sdc * p[c] + ct * amb;
+                }
+        double* tmp = cur; cur = nxt; nxt = tmp;
+    }
+    memcpy(out, cur, n * sizeof(double));
+    free(cur); free(nxt);
+    return ORACLE_OK;
+}
