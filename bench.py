@@ -286,6 +286,36 @@ def extra_workloads(rg, torch, tune: bool):
         out["srad_v1"] = res
     except Exception as e:  # noqa: BLE001
         out["srad_v1"] = {"error": str(e)[:200]}
+    # hotspot3D: Rodinia's 512 x 512 x 8 x 100 (L2-resident) and a
+    # 1024 x 1024 x 64 x 20 grid (HBM-resident, 12 B per cell-update roofline)
+    try:
+        import numpy as np
+        res = {}
+        for label, (nx, ny, nz, it) in (("rodinia_512x512x8", (512, 512, 8, 100)),
+                                        ("large_1024x1024x64", (1024, 1024, 64, 20))):
+            rng = np.random.default_rng(1)
+            T = torch.from_numpy((323.15 + 20 * rng.random((nz, ny, nx))).astype(np.float32)).cuda()
+            P = torch.from_numpy((1e-3 * rng.random((nz, ny, nx))).astype(np.float32)).cuda()
+            O = torch.empty_like(T)
+            S = torch.empty_like(T)
+            c = rg.rodinia_hotspot3d_coeffs_rodinia(nx, ny, nz)
+            r = {}
+            for name, g in (("uncoarsened", UNC), ("tuned", None)):
+                if name == "tuned" and tune:
+                    g, _ = rg.rodinia_tune("hotspot3d", ny, nx, it, reps=2, depth=nz)
+                ms = timed(lambda: rg.rodinia_hotspot3d(T, P, it, coeffs=c, g=g, out=O, scratch=S), reps=3)
+                ups = nx * ny * nz * it / (ms * 1e-3)
+                r[name] = {"ms": ms, "cell_updates_per_s": ups, "effective_GBps": 12 * ups / 1e9,
+                           "g": list(g.astuple()) if hasattr(g, "astuple") else (list(g) if g else None)}
+            r["speedup"] = r["uncoarsened"]["ms"] / r["tuned"]["ms"]
+            res[label] = r
+        hbm, src = _peaks()
+        ach = res["large_1024x1024x64"]["tuned"]["effective_GBps"]
+        res["roofline"] = {"bound": "hbm", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm,
+                           "bytes_per_update": 12, "config": "large_1024x1024x64", "peak_source": src}
+        out["hotspot3d"] = res
+    except Exception as e:  # noqa: BLE001
+        out["hotspot3d"] = {"error": str(e)[:200]}
     # pathfinder 100 rows x 100000 cols int32, per-call time over batches
     try:
         import synth

@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define RODINIA_ABI_VERSION 1
+#define RODINIA_ABI_VERSION 2
 
 typedef enum {
     RODINIA_OK = 0,
@@ -96,7 +96,9 @@ typedef struct {
 #define RODINIA_OCC(n) (((n) & 0xff) << 8)
 #define RODINIA_OCC_OF(flags) (((flags) >> 8) & 0xff)
 
-typedef enum { RODINIA_HOTSPOT = 0, RODINIA_SRAD = 1, RODINIA_PATHFINDER = 2, RODINIA_LUD = 3 } rodinia_kernel;
+typedef enum {
+    RODINIA_HOTSPOT = 0, RODINIA_SRAD = 1, RODINIA_PATHFINDER = 2, RODINIA_LUD = 3, RODINIA_HOTSPOT3D = 4
+} rodinia_kernel;
 
 /* ---------------------------------------------------------------------------------------
  * hotspot -- Rodinia hotspot `calculate_temp` (2-D thermal RC stencil), see DESIGN.md §3 H1-H8.
@@ -128,6 +130,31 @@ rodinia_status rodinia_hotspot_host(const float* temp_in, const float* power, fl
                                     int64_t rows, int64_t cols, int32_t iterations,
                                     const rodinia_hotspot_coeffs* coeffs,
                                     const rodinia_granularity* g, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * hotspot3d -- Rodinia hotspot3D `hotspotOpt1` (7-point 3-D thermal stencil, named in
+ * PAPER.md:395), readings T1-T4.  Grid nx (x, fastest) x ny x nz,
+ * index z*nx*ny + y*nx + x.  One step, every cell, neighbours clamped to the grid:
+ *   T' = cc*c + cw*W + ce*E + cs*S + cn*N + cb*B + ct*T + sdc*P + ct*amb
+ * (W/E: x-+1, N/S: y-+1, B/T: z-+1), summed left to right in fp32. */
+typedef struct { float cc, cw, ce, cs, cn, cb, ct, sdc, amb; } rodinia_hotspot3d_coeffs;
+
+/* Rodinia's chip formulas (fp64, rounded once): dx = chip_h/ny, dy = chip_w/nx, dz = t_chip/nz,
+ * sdc = dt/Cap, ce = cw = sdc/Rx, cn = cs = sdc/Ry, ct = cb = sdc/Rz, cc = 1 - (2ce+2cn+3ct). */
+rodinia_status rodinia_hotspot3d_coeffs_rodinia(int64_t nx, int64_t ny, int64_t nz, double chip_w_m,
+                                                double chip_h_m, double t_chip_m,
+                                                rodinia_hotspot3d_coeffs* out);
+
+/* `iterations` steps from temp_in (never written) into temp_out; power nx*ny*nz; scratch NULL or
+ * an nx*ny*nz buffer; coeffs NULL => Rodinia's 16 mm x 16 mm x 0.5 mm chip. */
+rodinia_status rodinia_hotspot3d(const float* temp_in, const float* power, float* temp_out,
+                                 float* scratch, int64_t nx, int64_t ny, int64_t nz,
+                                 int32_t iterations, const rodinia_hotspot3d_coeffs* coeffs,
+                                 const rodinia_granularity* g, void* stream);
+rodinia_status rodinia_hotspot3d_host(const float* temp_in, const float* power, float* temp_out,
+                                      int64_t nx, int64_t ny, int64_t nz, int32_t iterations,
+                                      const rodinia_hotspot3d_coeffs* coeffs,
+                                      const rodinia_granularity* g, void* stream);
 
 /* ---------------------------------------------------------------------------------------
  * srad_v2 -- Rodinia srad_v2 (speckle-reducing anisotropic diffusion), DESIGN.md §3 S1-S9.
@@ -180,10 +207,13 @@ rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel,
  * Variants, compile-time filter and timing-driven tuning (§VI, 251-269).
  */
 typedef struct {
-    int64_t rows, cols;      /* lud: rows = cols = n; pathfinder: rows x cols wall */
+    int64_t rows, cols;      /* lud: rows = cols = n; pathfinder: rows x cols wall;
+                                hotspot3d: rows = ny, cols = nx (depth = nz) */
     int32_t iterations;      /* hotspot / srad iterations (tuning times a prefix of them);
                                 lud: the panel width (0 => 16); pathfinder: unused */
     int32_t nranks;          /* 1 for single-GPU problems; part of the cache key */
+    int32_t depth;           /* hotspot3d: nz (0 => 1); others: 0 */
+    int32_t reserved;        /* 0 */
 } rodinia_problem;
 
 typedef struct {

@@ -40,8 +40,8 @@ RODINIA_E_NOMEM = -10
 RODINIA_FAITHFUL = 1
 RODINIA_STREAM = 2
 
-RODINIA_HOTSPOT, RODINIA_SRAD, RODINIA_PATHFINDER, RODINIA_LUD = 0, 1, 2, 3
-KERNELS = {"hotspot": 0, "srad": 1, "pathfinder": 2, "lud": 3}
+RODINIA_HOTSPOT, RODINIA_SRAD, RODINIA_PATHFINDER, RODINIA_LUD, RODINIA_HOTSPOT3D = 0, 1, 2, 3, 4
+KERNELS = {"hotspot": 0, "srad": 1, "pathfinder": 2, "lud": 3, "hotspot3d": 4}
 
 
 class RodiniaError(RuntimeError):
@@ -81,7 +81,12 @@ class HotspotCoeffs(ctypes.Structure):
 
 class Problem(ctypes.Structure):
     _fields_ = [("rows", ctypes.c_int64), ("cols", ctypes.c_int64),
-                ("iterations", ctypes.c_int32), ("nranks", ctypes.c_int32)]
+                ("iterations", ctypes.c_int32), ("nranks", ctypes.c_int32),
+                ("depth", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+
+
+class Hotspot3dCoeffs(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_float) for k in ("cc", "cw", "ce", "cs", "cn", "cb", "ct", "sdc", "amb")]
 
 
 class TuneRow(ctypes.Structure):
@@ -110,6 +115,9 @@ _SIGS = {
     "rodinia_hotspot_coeffs_rodinia": ([_i64, _i64, _f64, _f64, _PC], _i32),
     "rodinia_hotspot": ([_vp, _vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
     "rodinia_hotspot_host": ([_vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
+    "rodinia_hotspot3d_coeffs_rodinia": ([_i64, _i64, _i64, _f64, _f64, _f64, ctypes.c_void_p], _i32),
+    "rodinia_hotspot3d": ([_vp, _vp, _vp, _vp, _i64, _i64, _i64, _i32, _vp, _PG, _vp], _i32),
+    "rodinia_hotspot3d_host": ([_vp, _vp, _vp, _i64, _i64, _i64, _i32, _vp, _PG, _vp], _i32),
     "rodinia_srad": ([_vp, _i64, _i64, _i64, _i64, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
     "rodinia_srad_host": ([_vp, _i64, _i64, _i64, _i64, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
     "rodinia_srad_v1": ([_vp, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
@@ -235,6 +243,44 @@ def rodinia_hotspot_host(temp, power, iterations: int, coeffs=None, g=None, out=
     return out
 
 
+# ----------------------------------------------------------------------------- hotspot3d
+def rodinia_hotspot3d_coeffs_rodinia(nx: int, ny: int, nz: int, chip_w: float = 0.016, chip_h: float = 0.016,
+                                     t_chip: float = 0.0005) -> Hotspot3dCoeffs:
+    c = Hotspot3dCoeffs()
+    check(lib.rodinia_hotspot3d_coeffs_rodinia(nx, ny, nz, chip_w, chip_h, t_chip, ctypes.addressof(c)),
+          "rodinia_hotspot3d_coeffs_rodinia")
+    return c
+
+
+def rodinia_hotspot3d(temp, power, iterations: int, coeffs=None, g=None, out=None, scratch=None, stream=None):
+    """`iterations` hotspot3D steps of temp ((nz, ny, nx) float32 CUDA tensor); returns temp_out."""
+    import torch
+    if temp.dim() != 3 or power.shape != temp.shape:
+        raise ValueError("temp and power must be equal-shaped (nz, ny, nx) tensors")
+    nz, ny, nx = temp.shape
+    if out is None:
+        out = torch.empty_like(temp)
+    check(lib.rodinia_hotspot3d(_dev(temp, torch.float32, "temp"), _dev(power, torch.float32, "power"),
+                                _dev(out, torch.float32, "out"),
+                                None if scratch is None else _dev(scratch, torch.float32, "scratch"),
+                                nx, ny, nz, int(iterations), None if coeffs is None else ctypes.addressof(coeffs),
+                                _g(g), _stream(stream)), "rodinia_hotspot3d")
+    return out
+
+
+def rodinia_hotspot3d_host(temp, power, iterations: int, coeffs=None, g=None, stream=None):
+    import numpy as np
+    t = np.ascontiguousarray(temp, dtype=np.float32)
+    p = np.ascontiguousarray(power, dtype=np.float32)
+    out = np.empty_like(t)
+    nz, ny, nx = t.shape
+    check(lib.rodinia_hotspot3d_host(ctypes.c_void_p(t.ctypes.data), ctypes.c_void_p(p.ctypes.data),
+                                     ctypes.c_void_p(out.ctypes.data), nx, ny, nz, int(iterations),
+                                     None if coeffs is None else ctypes.addressof(coeffs), _g(g), _stream(stream)),
+          "rodinia_hotspot3d_host")
+    return out
+
+
 # ----------------------------------------------------------------------------- srad
 def rodinia_srad(J, r1, r2, c1, c2, lam: float, niter: int, g=None, stream=None):
     """niter srad_v2 iterations on J (R x C float32 CUDA tensor, in place); returns J."""
@@ -327,9 +373,10 @@ def rodinia_variants(kernel):
     return [rows[i].asdict() for i in range(n.value)]
 
 
-def rodinia_tune(kernel, rows: int, cols: int, iterations: int = 1, nranks: int = 1, reps: int = 3):
+def rodinia_tune(kernel, rows: int, cols: int, iterations: int = 1, nranks: int = 1, reps: int = 3,
+                 depth: int = 0):
     """Timing-driven selection. Returns (best Granularity, [row dicts])."""
-    p = Problem(rows, cols, iterations, nranks)
+    p = Problem(rows, cols, iterations, nranks, depth, 0)
     best = Granularity()
     cap = _i32(4096)
     out = (TuneRow * cap.value)()
@@ -338,8 +385,8 @@ def rodinia_tune(kernel, rows: int, cols: int, iterations: int = 1, nranks: int 
     return best, [out[i].asdict() for i in range(min(cap.value, 4096))]
 
 
-def rodinia_resolve(kernel, rows: int, cols: int, iterations: int = 1, nranks: int = 1):
-    p = Problem(rows, cols, iterations, nranks)
+def rodinia_resolve(kernel, rows: int, cols: int, iterations: int = 1, nranks: int = 1, depth: int = 0):
+    p = Problem(rows, cols, iterations, nranks, depth, 0)
     g = Granularity()
     check(lib.rodinia_resolve(_kernel(kernel), ctypes.byref(p), ctypes.byref(g)), "rodinia_resolve")
     return g

@@ -137,8 +137,8 @@ static std::string cache_key(rodinia_kernel k, const rodinia_problem& p) {
     const char* dev = "nodev";
     int sms = 0;
     if (device_info(&di) == RODINIA_OK) { dev = di.name; sms = di.sms; }
-    snprintf(b, sizeof b, "%s|%d|%d|%lldx%lld|%d|%d", dev, sms, (int)k, (long long)p.rows,
-             (long long)p.cols, p.iterations, p.nranks);
+    snprintf(b, sizeof b, "%s|%d|%d|%lldx%lldx%d|%d|%d", dev, sms, (int)k, (long long)p.rows,
+             (long long)p.cols, p.depth, p.iterations, p.nranks);
     return b;
 }
 

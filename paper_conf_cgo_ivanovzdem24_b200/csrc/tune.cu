@@ -47,6 +47,8 @@ int pathfinder_num_variants();
 void pathfinder_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
 int lud_num_variants();
 void lud_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
+int hotspot3d_num_variants();
+void hotspot3d_variant_info(int, rodinia_granularity*, const void**, const char**, int*);
 
 static Registry registry(rodinia_kernel k) {
     switch (k) {
@@ -54,6 +56,7 @@ static Registry registry(rodinia_kernel k) {
         case RODINIA_SRAD: return {srad_num_variants, srad_variant_info};
         case RODINIA_PATHFINDER: return {pathfinder_num_variants, pathfinder_variant_info};
         case RODINIA_LUD: return {lud_num_variants, lud_variant_info};
+        case RODINIA_HOTSPOT3D: return {hotspot3d_num_variants, hotspot3d_variant_info};
     }
     return {nullptr, nullptr};
 }
@@ -99,6 +102,7 @@ rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
             return gran(4, 1, 1, 1, 1, 1);
         case RODINIA_SRAD: return gran(4, 1, 1, 2, 1, 1, RODINIA_STREAM);
         case RODINIA_PATHFINDER: return gran(4, 1, 1, 1, 8, 1);
+        case RODINIA_HOTSPOT3D: return gran(4, 1, 1, 1, 1, 1);
         case RODINIA_LUD:  // measured on B200 at n = 8192
             return p.iterations == 32 ? gran(2, 4, 4, 2, 1, 1) : gran(4, 2, 2, 2, 1, 1);
     }
@@ -273,6 +277,7 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
 rodinia_status tune_srad(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
 rodinia_status tune_pathfinder(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
 rodinia_status tune_lud(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
+rodinia_status tune_hotspot3d(const rodinia_problem& p, int reps, rodinia_granularity* best, std::vector<rodinia_tune_row>* rows);
 
 }  // namespace rg
 
@@ -280,7 +285,7 @@ using namespace rg;
 
 extern "C" rodinia_status rodinia_variants(rodinia_kernel k, rodinia_tune_row* out, int32_t* n) {
     if (!n || *n < 0 || (*n > 0 && !out)) return set_error(RODINIA_E_INVALID, "variants: bad arguments");
-    if ((int)k < 0 || (int)k > 3) return set_error(RODINIA_E_INVALID, "variants: unknown kernel %d", (int)k);
+    if ((int)k < 0 || (int)k > 4) return set_error(RODINIA_E_INVALID, "variants: unknown kernel %d", (int)k);
     Registry reg = registry(k);
     const int total = reg.count();
     int cnt = 0;
@@ -298,7 +303,7 @@ extern "C" rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* 
     if (!p || !best || reps < 1 || p->rows < 1 || p->cols < 1 || p->iterations < 0 || p->nranks < 1)
         return set_error(RODINIA_E_INVALID, "tune: bad arguments");
     if (nrows && *nrows > 0 && !rows) return set_error(RODINIA_E_INVALID, "tune: rows is null");
-    if ((int)k < 0 || (int)k > 3) return set_error(RODINIA_E_INVALID, "tune: unknown kernel %d", (int)k);
+    if ((int)k < 0 || (int)k > 4) return set_error(RODINIA_E_INVALID, "tune: unknown kernel %d", (int)k);
     DeviceInfo di;
     RG_TRY(device_info(&di));
     std::vector<rodinia_tune_row> out;
@@ -307,6 +312,7 @@ extern "C" rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* 
         case RODINIA_HOTSPOT: st = tune_hotspot(*p, reps, best, &out); break;
         case RODINIA_SRAD: st = tune_srad(*p, reps, best, &out); break;
         case RODINIA_PATHFINDER: st = tune_pathfinder(*p, reps, best, &out); break;
+        case RODINIA_HOTSPOT3D: st = tune_hotspot3d(*p, reps, best, &out); break;
         default: st = tune_lud(*p, reps, best, &out); break;
     }
     if (nrows) {

@@ -1,0 +1,93 @@
+"""GPU parity of hotspot3D against the fp64 oracle; all variants bitwise equal."""
+import numpy as np
+import pytest
+
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-5
+UNC = (1, 1, 1, 1, 1, 0, 0)
+
+
+@pytest.fixture(scope="module")
+def rg():
+    import paper_conf_cgo_ivanovzdem24_b200 as m
+    return m
+
+
+def _inputs(nz, ny, nx, seed=1):
+    rng = np.random.default_rng(seed)
+    t = (323.15 + 20 * rng.random((nz, ny, nx))).astype(np.float32)
+    p = (1e-3 * rng.random((nz, ny, nx))).astype(np.float32)
+    return t, p
+
+
+def _coef(rg, nx, ny, nz):
+    c = rg.rodinia_hotspot3d_coeffs_rodinia(nx, ny, nz)
+    return c, {k: float(getattr(c, k)) for k in oracle.HS3D_KEYS}
+
+
+def _run(rg, T, P, iters, c, g):
+    out = rg.rodinia_hotspot3d(torch.from_numpy(T).cuda(), torch.from_numpy(P).cuda(), iters, coeffs=c, g=g)
+    torch.cuda.synchronize()
+    return out.cpu().numpy()
+
+
+def _rel(a, b):
+    return float(np.max(np.abs(a.astype(np.float64) - b) / np.abs(b)))
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (1, 5, 70), (8, 8, 8), (3, 37, 130), (8, 64, 64)])
+def test_vs_oracle(rg, shape):
+    nz, ny, nx = shape
+    T, P = _inputs(*shape)
+    c, cd = _coef(rg, nx, ny, nz)
+    ocf = oracle.hotspot3d_coeffs(nx, ny, nz)
+    for k in oracle.HS3D_KEYS:  # the library's coefficients are the oracle's rounded once
+        assert cd[k] == np.float32(ocf[k])
+    for iters in (0, 1, 5):
+        for g in (UNC, (4, 1, 2, 1, 1, 1, 0)):
+            assert _rel(_run(rg, T, P, iters, c, g), oracle.hotspot3d(T, P, iters, cd)) <= TOL, (shape, iters, g)
+
+
+def test_rodinia_config_512x512x8_100_iterations(rg):
+    T, P = _inputs(8, 512, 512, seed=2)
+    c, cd = _coef(rg, 512, 512, 8)
+    got = _run(rg, T, P, 100, c, None)
+    assert _rel(got, oracle.hotspot3d(T, P, 100, cd)) <= TOL
+    assert np.array_equal(got, _run(rg, T, P, 100, c, UNC))
+
+
+def test_all_variants_bit_identical(rg):
+    T, P = _inputs(5, 45, 200, seed=3)
+    c, cd = _coef(rg, 200, 45, 5)
+    base = _run(rg, T, P, 7, c, UNC)
+    for r in rg.rodinia_variants("hotspot3d"):
+        g = r["g"]
+        for bx, by in [(1, 1), (3, 2)]:
+            gg = (g[0], g[1], bx, by, 1, g[5], 0)
+            assert np.array_equal(_run(rg, T, P, 7, c, gg), base), gg
+
+
+def test_ambient_fixed_point_and_host(rg):
+    T = np.full((4, 30, 50), 80.0, np.float32)
+    c, cd = _coef(rg, 50, 30, 4)
+    out = _run(rg, T, np.zeros_like(T), 20, c, (2, 2, 1, 1, 1, 1, 0))
+    # the fp32-rounded coefficients do not sum to exactly 1, so the ambient state drifts by
+    # O(1e-7) per step in any precision that uses them; parity is against the oracle run with
+    # the same coefficients, and the drift stays small
+    assert _rel(out, oracle.hotspot3d(T, np.zeros_like(T), 20, cd)) <= TOL
+    assert _rel(out, T) <= 1e-5
+    T2, P2 = _inputs(4, 30, 50, seed=4)
+    got = rg.rodinia_hotspot3d_host(T2, P2, 6, coeffs=c, g=(4, 1, 1, 1, 1, 1, 0))
+    assert _rel(got, oracle.hotspot3d(T2, P2, 6, cd)) <= TOL
+
+
+def test_tune(rg):
+    best, rows = rg.rodinia_tune("hotspot3d", 256, 256, 10, reps=1, depth=8)
+    assert any(r["status"] == 0 for r in rows)
+    T, P = _inputs(8, 256, 256, seed=5)
+    c, cd = _coef(rg, 256, 256, 8)
+    assert np.array_equal(_run(rg, T, P, 10, c, best), _run(rg, T, P, 10, c, UNC))
