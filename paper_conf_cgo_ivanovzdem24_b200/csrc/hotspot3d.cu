@@ -93,6 +93,114 @@ __global__ void __launch_bounds__((64 / TX) * (4 / TY))
         }
 }
 
+// h3_plane<TX,TY> (flags RODINIA_STREAM): 2.5-D blocking for B200.  A 256-thread CTA owns a
+// (32*TX) x (8*TY) tile of (x, y) columns and marches z; each thread keeps its TX x TY cells'
+// values at z-1, z, z+1 in registers (B, C, T) and publishes C through a double-buffered
+// shared-memory plane whose one-cell halo ring is read from global memory with clamped indices
+// (which reproduces the clamped boundary), so N/S/E/W come from shared memory and each plane
+// costs one barrier.  HBM per cell-update: T read once (+ halo re-reads from L2), P read, T'
+// written.  TX % 4 == 0 moves rows with 128-bit accesses.
+template <int TX, int TY>
+__global__ void __launch_bounds__(256)
+    h3_plane(const float* __restrict__ tin, const float* __restrict__ pw, float* __restrict__ tout, int nx,
+             int ny, int nz, int bx, int by, H3Coef k) {
+    constexpr int OX = 32 * TX, OY = 8 * TY, SX = OX + 2, SY = OY + 2;
+    __shared__ float pl[2][SY][SX + 1];
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    const size_t plane = (size_t)nx * ny;
+    const bool vec = (TX % 4 == 0) && ((nx & 3) == 0);
+    (void)bx; (void)by;
+    const int x0 = blockIdx.x * OX, y0 = blockIdx.y * OY;
+    int xs[TX], ys[TY];
+#pragma unroll
+    for (int i = 0; i < TX; ++i) xs[i] = min(x0 + tx * TX + i, nx - 1);
+#pragma unroll
+    for (int j = 0; j < TY; ++j) ys[j] = min(y0 + ty * TY + j, ny - 1);
+    const bool full_x = x0 + tx * TX + TX <= nx;
+    auto load_cells = [&](int z, float (&v)[TY][TX], const float* __restrict__ base) {
+        const float* pz = base + (size_t)z * plane;
+#pragma unroll
+        for (int j = 0; j < TY; ++j) {
+            const float* row = pz + (size_t)ys[j] * nx;
+            if (vec && full_x) {
+#pragma unroll
+                for (int q = 0; q < TX / 4; ++q) {
+                    const float4 t = __ldg(reinterpret_cast<const float4*>(row + x0 + tx * TX) + q);
+                    v[j][(4 * q) % TX] = t.x; v[j][(4 * q + 1) % TX] = t.y;
+                    v[j][(4 * q + 2) % TX] = t.z; v[j][(4 * q + 3) % TX] = t.w;
+                }
+            } else {
+#pragma unroll
+                for (int i = 0; i < TX; ++i) v[j][i] = __ldg(row + xs[i]);
+            }
+        }
+    };
+    float B[TY][TX], Cc[TY][TX], T[TY][TX];
+    load_cells(0, Cc, tin);
+#pragma unroll
+    for (int j = 0; j < TY; ++j)
+#pragma unroll
+        for (int i = 0; i < TX; ++i) B[j][i] = Cc[j][i];
+    load_cells(min(1, nz - 1), T, tin);
+    // halo ring of the tile: left/right columns (SY cells each) and top/bottom rows (OX each)
+    const int nhalo = 2 * SY + 2 * OX;
+    for (int z = 0; z < nz; ++z) {
+        const int buf = z & 1;
+        const float* pz = tin + (size_t)z * plane;
+#pragma unroll
+        for (int j = 0; j < TY; ++j)
+#pragma unroll
+            for (int i = 0; i < TX; ++i) pl[buf][1 + ty * TY + j][1 + tx * TX + i] = Cc[j][i];
+        for (int h = threadIdx.x; h < nhalo; h += 256) {
+            int sy, sx;
+            if (h < SY) { sy = h; sx = 0; }
+            else if (h < 2 * SY) { sy = h - SY; sx = SX - 1; }
+            else if (h < 2 * SY + OX) { sy = 0; sx = 1 + (h - 2 * SY); }
+            else { sy = SY - 1; sx = 1 + (h - 2 * SY - OX); }
+            const int gy = min(max(y0 - 1 + sy, 0), ny - 1), gx = min(max(x0 - 1 + sx, 0), nx - 1);
+            pl[buf][sy][sx] = __ldg(pz + (size_t)gy * nx + gx);
+        }
+        float P[TY][TX];
+        load_cells(z, P, pw);
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < TY; ++j) {
+            const int ly = 1 + ty * TY + j;
+            const int gy = y0 + ty * TY + j;
+            float o[TX];
+#pragma unroll
+            for (int i = 0; i < TX; ++i) {
+                const int lx = 1 + tx * TX + i;
+                // clamped halo / interior values; cells beyond the grid edge hold clamped copies
+                const float w = (x0 + tx * TX + i == 0) ? Cc[j][i] : pl[buf][ly][lx - 1];
+                const float e = (x0 + tx * TX + i >= nx - 1) ? Cc[j][i] : pl[buf][ly][lx + 1];
+                const float n = (gy == 0) ? Cc[j][i] : pl[buf][ly - 1][lx];
+                const float s_ = (gy >= ny - 1) ? Cc[j][i] : pl[buf][ly + 1][lx];
+                o[i] = h3_cell(Cc[j][i], w, e, s_, n, B[j][i], T[j][i], P[j][i], k);
+            }
+            if (gy < ny) {
+                float* orow = tout + (size_t)z * plane + (size_t)gy * nx;
+                if (vec && full_x) {
+#pragma unroll
+                    for (int q = 0; q < TX / 4; ++q)
+                        reinterpret_cast<float4*>(orow + x0 + tx * TX)[q] =
+                            make_float4(o[(4 * q) % TX], o[(4 * q + 1) % TX], o[(4 * q + 2) % TX], o[(4 * q + 3) % TX]);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < TX; ++i)
+                        if (x0 + tx * TX + i < nx) orow[x0 + tx * TX + i] = o[i];
+                }
+            }
+        }
+        // advance the z window (T of plane z+2, clamped)
+#pragma unroll
+        for (int j = 0; j < TY; ++j)
+#pragma unroll
+            for (int i = 0; i < TX; ++i) { B[j][i] = Cc[j][i]; Cc[j][i] = T[j][i]; }
+        if (z + 1 < nz) load_cells(min(z + 2, nz - 1), T, tin);
+    }
+}
+
 namespace hotspot3d {
 
 typedef void (*Fn)(const float*, const float*, float*, int, int, int, int, int, H3Coef);
@@ -106,7 +214,19 @@ static const Variant kVariants[] = {
 #undef RG_H32
 #undef RG_H3
 
-static const Variant* find(int tx, int ty, int mode) {
+static const Variant kPlane[] = {
+    {1, 1, 1, h3_plane<1, 1>, "void rg::h3_plane<1, 1>"}, {2, 1, 1, h3_plane<2, 1>, "void rg::h3_plane<2, 1>"},
+    {4, 1, 1, h3_plane<4, 1>, "void rg::h3_plane<4, 1>"}, {4, 2, 1, h3_plane<4, 2>, "void rg::h3_plane<4, 2>"},
+    {2, 2, 1, h3_plane<2, 2>, "void rg::h3_plane<2, 2>"}, {1, 4, 1, h3_plane<1, 4>, "void rg::h3_plane<1, 4>"},
+    {4, 4, 1, h3_plane<4, 4>, "void rg::h3_plane<4, 4>"},
+};
+
+static const Variant* find(int tx, int ty, int mode, bool plane) {
+    if (plane) {
+        for (const auto& v : kPlane)
+            if (v.tx == tx && v.ty == ty) return &v;
+        return nullptr;
+    }
     for (const auto& v : kVariants)
         if (v.tx == tx && v.ty == ty && v.mode == mode) return &v;
     return nullptr;
@@ -116,18 +236,34 @@ rodinia_status check(const rodinia_granularity& g, int64_t ny, const Variant** o
     if (g.thread_x < 1 || g.thread_y < 1 || g.block_x < 1 || g.block_y < 1 || g.temporal != 1)
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: factors >= 1, temporal = 1 (%s)", gran_str(g).c_str());
     if (g.index_mode != 0 && g.index_mode != 1) return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: index_mode 0/1");
-    if (64 % g.thread_x || 4 % g.thread_y)
-        return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: thread factors must divide the 64 x 4 tile (PAPER.md:237)");
-    if (g.flags & RODINIA_STREAM) return set_error(RODINIA_E_NOT_BUILT, "hotspot3d: no stream family");
-    if (((ny + 3) / 4 + g.block_y - 1) / g.block_y > 65535)
-        return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: grid.y too large; raise block_y");
-    *out = find(g.thread_x, g.thread_y, g.index_mode);
+    const bool plane = (g.flags & RODINIA_STREAM) != 0;
+    if (plane) {
+        if (g.block_x != 1 || g.block_y != 1 || g.index_mode != 1)
+            return set_error(RODINIA_E_NOT_BUILT, "hotspot3d: the plane family has block factors 1, index_mode 1");
+        if ((ny + 8 * g.thread_y - 1) / (8 * g.thread_y) > 65535)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: grid.y too large");
+    } else {
+        if (64 % g.thread_x || 4 % g.thread_y)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: thread factors must divide the 64 x 4 tile (PAPER.md:237)");
+        if (((ny + 3) / 4 + g.block_y - 1) / g.block_y > 65535)
+            return set_error(RODINIA_E_ILLEGAL_FACTOR, "hotspot3d: grid.y too large; raise block_y");
+    }
+    *out = find(g.thread_x, g.thread_y, g.index_mode, plane);
     if (!*out) return set_error(RODINIA_E_NOT_BUILT, "hotspot3d: variant %s not instantiated", gran_str(g).c_str());
     return RODINIA_OK;
 }
 
-int num_variants() { return (int)(sizeof(kVariants) / sizeof(kVariants[0])); }
+int num_variants() { return (int)(sizeof(kVariants) / sizeof(kVariants[0]) + sizeof(kPlane) / sizeof(kPlane[0])); }
 void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    const int nd = (int)(sizeof(kVariants) / sizeof(kVariants[0]));
+    if (i >= nd) {
+        const auto& v = kPlane[i - nd];
+        *g = gran(v.tx, v.ty, 1, 1, 1, 1, RODINIA_STREAM);
+        *fn = (const void*)v.fn;
+        *key = v.key;
+        *threads = 256;
+        return;
+    }
     const auto& v = kVariants[i];
     *g = gran(v.tx, v.ty, 1, 1, 1, v.mode);
     *fn = (const void*)v.fn;
@@ -142,8 +278,13 @@ rodinia_status run(const float* tin, const float* p, float* tout, float* scr, in
         RG_CUDA(cudaMemcpyAsync(tout, tin, n * sizeof(float), cudaMemcpyDeviceToDevice, s));
         return RODINIA_OK;
     }
-    dim3 grid(((nx + 63) / 64 + bx - 1) / bx, ((ny + 3) / 4 + by - 1) / by);
-    dim3 block(64 / v->tx, 4 / v->ty);
+    const bool plane = v->mode == 1 && (v->fn == (Fn)h3_plane<1, 1> || v->fn == (Fn)h3_plane<2, 1> ||
+                                         v->fn == (Fn)h3_plane<4, 1> || v->fn == (Fn)h3_plane<4, 2> ||
+                                         v->fn == (Fn)h3_plane<2, 2> || v->fn == (Fn)h3_plane<1, 4> ||
+                                         v->fn == (Fn)h3_plane<4, 4>);
+    dim3 grid = plane ? dim3((nx + 32 * v->tx - 1) / (32 * v->tx), (ny + 8 * v->ty - 1) / (8 * v->ty))
+                      : dim3(((nx + 63) / 64 + bx - 1) / bx, ((ny + 3) / 4 + by - 1) / by);
+    dim3 block = plane ? dim3(256) : dim3(64 / v->tx, 4 / v->ty);
     const float* src = tin;
     for (int l = 0; l < iters; ++l) {
         float* dst = ((iters - 1 - l) % 2 == 0) ? tout : scr;
@@ -280,6 +421,7 @@ rodinia_status tune_hotspot3d(const rodinia_problem& pr, int reps, rodinia_granu
     for (int vi = 0; st == RODINIA_OK && vi < hotspot3d::num_variants(); ++vi) {
         for (auto b : {std::make_pair(1, 1), std::make_pair(2, 1), std::make_pair(1, 2), std::make_pair(2, 2),
                        std::make_pair(1, 4)}) {
+            if (vi >= (int)(sizeof(hotspot3d::kVariants) / sizeof(hotspot3d::kVariants[0])) && (b.first != 1 || b.second != 1)) continue;
             rodinia_tune_row row;
             memset(&row, 0, sizeof row);
             const void* fn;

@@ -64,11 +64,21 @@ def test_all_variants_bit_identical(rg):
     T, P = _inputs(5, 45, 200, seed=3)
     c, cd = _coef(rg, 200, 45, 5)
     base = _run(rg, T, P, 7, c, UNC)
+    seen_plane = False
     for r in rg.rodinia_variants("hotspot3d"):
         g = r["g"]
-        for bx, by in [(1, 1), (3, 2)]:
-            gg = (g[0], g[1], bx, by, 1, g[5], 0)
+        plane = bool(g[6] & rg.RODINIA_STREAM)
+        seen_plane |= plane
+        for bx, by in ([(1, 1)] if plane else [(1, 1), (3, 2)]):
+            gg = (g[0], g[1], bx, by, 1, g[5], g[6])
             assert np.array_equal(_run(rg, T, P, 7, c, gg), base), gg
+    assert seen_plane
+    # a shape where the plane tiles are ragged in x and y and nz = 2
+    T2, P2 = _inputs(2, 19, 141, seed=7)
+    c2, _ = _coef(rg, 141, 19, 2)
+    b2 = _run(rg, T2, P2, 5, c2, UNC)
+    for g in [(4, 1, 1, 1, 1, 1, 2), (1, 4, 1, 1, 1, 1, 2), (4, 4, 1, 1, 1, 1, 2)]:
+        assert np.array_equal(_run(rg, T2, P2, 5, c2, g), b2), g
 
 
 def test_ambient_fixed_point_and_host(rg):
