@@ -261,6 +261,100 @@ __global__ void __launch_bounds__((P / TX) * (P / TY),
     }
 }
 
+// ------------------------------------------------------------------ streaming trailing update
+// lud_internal_stream<P,V> (flags RODINIA_STREAM): column-stationary update for B200.  A CTA of
+// 256 threads owns 256*V contiguous trailing columns and a chunk of 16*by rows; each thread keeps
+// its V columns of U12 (P x V values) in registers, the chunk's L21 rows are staged in shared
+// memory (read by broadcast), and A streams through once: one 128-bit load and one store per V
+// elements, A rows requested two rows ahead.  Per element the arithmetic is the same sequence as
+// every other variant (sum_i l_i u_i ascending with fma, then a -= sum), so results are
+// bit-identical for a fixed panel width.  Bound: HBM (8 B per element per step) at P = 16.
+template <int P, int V>
+__global__ void __launch_bounds__(256)
+    lud_internal_stream(float* const* __restrict__ slot, int n, int k, int chunk_tiles, int unused) {
+    float* A = *slot;
+    extern __shared__ __align__(16) float Lst[];  // [rows][P]
+    (void)unused;
+    const int o = k * P, t0 = o + P;
+    const int cbase = t0 + blockIdx.x * 256 * V + threadIdx.x * V;
+    const int r0 = t0 + blockIdx.y * chunk_tiles * 16;
+    const int r1 = min(n, r0 + chunk_tiles * 16);
+    if (r0 >= n) return;
+    // stage L21 rows of the chunk (row-major P values each)
+    for (int e = threadIdx.x; e < (r1 - r0) * P; e += 256) {
+        const int rr = e / P, i = e - rr * P;
+        Lst[e] = A[(size_t)(r0 + rr) * n + o + i];
+    }
+    // this thread's U12 columns
+    float u[P][V];
+    const bool vec = (V % 4 == 0) && ((n & 3) == 0) && cbase + V <= n;
+#pragma unroll
+    for (int i = 0; i < P; ++i) {
+        const float* urow = A + (size_t)(o + i) * n;
+        if (vec) {
+#pragma unroll
+            for (int q = 0; q < V / 4; ++q) {
+                const float4 t = *reinterpret_cast<const float4*>(urow + cbase + 4 * q);
+                u[i][4 * q] = t.x; u[i][(4 * q + 1) % V] = t.y; u[i][(4 * q + 2) % V] = t.z; u[i][(4 * q + 3) % V] = t.w;
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v) u[i][v] = cbase + v < n ? urow[cbase + v] : 0.f;
+        }
+    }
+    __syncthreads();
+    if (cbase >= n) return;
+    auto ld = [&](int r, float (&a)[V]) {
+        const float* row = A + (size_t)r * n;
+        if (vec) {
+#pragma unroll
+            for (int q = 0; q < V / 4; ++q) {
+                const float4 t = *reinterpret_cast<const float4*>(row + cbase + 4 * q);
+                a[4 * q] = t.x; a[(4 * q + 1) % V] = t.y; a[(4 * q + 2) % V] = t.z; a[(4 * q + 3) % V] = t.w;
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v) a[v] = cbase + v < n ? row[cbase + v] : 0.f;
+        }
+    };
+    float a0[V], a1[V];
+    ld(r0, a0);
+    if (r0 + 1 < r1) ld(r0 + 1, a1);
+    for (int r = r0; r < r1; ++r) {
+        float a2[V];
+        if (r + 2 < r1) ld(r + 2, a2);
+        const float* l = Lst + (r - r0) * P;
+        float sum[V];
+#pragma unroll
+        for (int v = 0; v < V; ++v) sum[v] = 0.f;
+#pragma unroll
+        for (int i4 = 0; i4 < P / 4; ++i4) {
+            const float4 l4 = reinterpret_cast<const float4*>(l)[i4];
+            const float lv[4] = {l4.x, l4.y, l4.z, l4.w};
+#pragma unroll
+            for (int ii = 0; ii < 4; ++ii)
+#pragma unroll
+                for (int v = 0; v < V; ++v) sum[v] = __fmaf_rn(lv[ii], u[4 * i4 + ii][v], sum[v]);
+        }
+        float res[V];
+#pragma unroll
+        for (int v = 0; v < V; ++v) res[v] = __fsub_rn(a0[v], sum[v]);
+        float* row = A + (size_t)r * n;
+        if (vec) {
+#pragma unroll
+            for (int q = 0; q < V / 4; ++q)
+                reinterpret_cast<float4*>(row + cbase)[q] =
+                    make_float4(res[4 * q], res[(4 * q + 1) % V], res[(4 * q + 2) % V], res[(4 * q + 3) % V]);
+        } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v)
+                if (cbase + v < n) row[cbase + v] = res[v];
+        }
+#pragma unroll
+        for (int v = 0; v < V; ++v) { a0[v] = a1[v]; a1[v] = a2[v]; }
+    }
+}
+
 __global__ void lud_set_slot(float** slot, float* a) { *slot = a; }
 
 namespace lud {
@@ -288,9 +382,18 @@ static const Variant* find(int p, int tx, int ty, int mode) {
     return nullptr;
 }
 
+struct StreamVariant { int p, v; IntFn fn; const char* key; };
+static const StreamVariant kStreamInt[] = {
+    {16, 4, lud_internal_stream<16, 4>, "void rg::lud_internal_stream<16, 4>"},
+    {16, 8, lud_internal_stream<16, 8>, "void rg::lud_internal_stream<16, 8>"},
+    {32, 2, lud_internal_stream<32, 2>, "void rg::lud_internal_stream<32, 2>"},
+    {32, 4, lud_internal_stream<32, 4>, "void rg::lud_internal_stream<32, 4>"},
+};
+
 struct Plan {
     int p;
     const Variant* v;
+    const StreamVariant* sv;  // streaming trailing update (flags & RODINIA_STREAM)
     int bx, by;
     size_t smem;
 };
@@ -303,9 +406,23 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: factors must be >= 1, temporal = 1 (%s)", gran_str(g).c_str());
     if (g.index_mode != 0 && g.index_mode != 1)
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: index_mode must be 0 or 1");
+    pl->sv = nullptr;
+    if (g.flags & RODINIA_STREAM) {
+        if (g.thread_y != 1 || g.index_mode != 1 || (g.flags & RODINIA_FAITHFUL))
+            return set_error(RODINIA_E_NOT_BUILT, "lud: stream family needs thread_y = 1, index_mode = 1");
+        for (const auto& x : kStreamInt)
+            if (x.p == panel && x.v == g.thread_x) pl->sv = &x;
+        if (!pl->sv) return set_error(RODINIA_E_NOT_BUILT, "lud: stream variant P=%d V=%d not built", panel, g.thread_x);
+        pl->p = panel;
+        pl->v = nullptr;
+        pl->bx = 1;
+        pl->by = g.block_y;  // rows per CTA in 16-row tiles
+        pl->smem = (size_t)16 * g.block_y * panel * sizeof(float);
+        if (pl->smem > 227 * 1024) return set_error(RODINIA_E_SMEM, "lud: stream chunk needs %zu B shared memory", pl->smem);
+        return RODINIA_OK;
+    }
     if (panel % g.thread_x || panel % g.thread_y)
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: thread factors must divide the %dx%d tile (PAPER.md:237)", panel, panel);
-    if (g.flags & RODINIA_STREAM) return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: no stream family");
     pl->p = panel;
     pl->v = find(panel, g.thread_x, g.thread_y, g.index_mode);
     if (!pl->v) return set_error(RODINIA_E_NOT_BUILT, "lud: internal variant P=%d %s not instantiated", panel, gran_str(g).c_str());
@@ -327,6 +444,12 @@ static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
         if (k == m - 1) break;
         perim<<<m - k - 1, 2 * P, 0, s>>>(slot, n, k);
         const int rem = m - k - 1;
+        if (pl.sv) {
+            const int width = n - P * (k + 1);
+            dim3 grid((width + 256 * pl.sv->v - 1) / (256 * pl.sv->v), (width + 16 * pl.by - 1) / (16 * pl.by));
+            pl.sv->fn<<<grid, 256, pl.smem, s>>>(slot, n, k, pl.by, 0);
+            continue;
+        }
         dim3 grid((rem + pl.bx - 1) / pl.bx, (rem + pl.by - 1) / pl.by);
         dim3 block(P / pl.v->tx, P / pl.v->ty);
         pl.v->fn<<<grid, block, pl.smem, s>>>(slot, n, k, pl.bx, pl.by);
@@ -344,14 +467,16 @@ static std::map<std::tuple<int, int, int, int, int, int, int, int, int>, GraphEn
 rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
     int dev = 0;
     RG_CUDA(cudaGetDevice(&dev));
-    const auto key = std::make_tuple(dev, n, pl.p, pl.v->tx, pl.v->ty, pl.v->mode, pl.bx, pl.by, 0);
+    const auto key = pl.sv ? std::make_tuple(dev, n, pl.p, pl.sv->v, 0, 1, pl.bx, pl.by, 1)
+                           : std::make_tuple(dev, n, pl.p, pl.v->tx, pl.v->ty, pl.v->mode, pl.bx, pl.by, 0);
     std::lock_guard<std::mutex> lk(g_mu);
     GraphEntry& ge = g_graphs[key];
     const int m = (n + pl.p - 1) / pl.p;
     if (!ge.exec) {
         RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
+        const void* ifn = pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
         if (pl.smem > 48 * 1024)
-            RG_CUDA(cudaFuncSetAttribute((const void*)pl.v->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
+            RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
         cudaStream_t cs;
         RG_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
         cudaGraph_t graph;
@@ -371,8 +496,17 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
     return RODINIA_OK;
 }
 
-int num_variants() { return (int)(sizeof(kInternal) / sizeof(kInternal[0])); }
+int num_variants() { return (int)(sizeof(kInternal) / sizeof(kInternal[0]) + sizeof(kStreamInt) / sizeof(kStreamInt[0])); }
 void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads) {
+    const int ni = (int)(sizeof(kInternal) / sizeof(kInternal[0]));
+    if (i >= ni) {
+        const auto& v = kStreamInt[i - ni];
+        *g = gran(v.v, 1, 1, 16, 1, 1, RODINIA_STREAM);
+        *fn = (const void*)v.fn;
+        *key = v.key;
+        *threads = 256;
+        return;
+    }
     const auto& v = kInternal[i];
     *g = gran(v.tx, v.ty, 1, 1, 1, v.mode);
     *fn = (const void*)v.fn;
@@ -433,9 +567,12 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
         const char* key;
         int threads;
         lud::variant_info(vi, &g0, &fn, &key, &threads);
-        if (lud::kInternal[vi].p != panel) continue;
+        const int ni = (int)(sizeof(lud::kInternal) / sizeof(lud::kInternal[0]));
+        const bool is_stream = vi >= ni;
+        if ((is_stream ? lud::kStreamInt[vi - ni].p : lud::kInternal[vi].p) != panel) continue;
         for (int bx : {1, 2, 4, 7})
-            for (int by : {1, 2, 4}) {
+            for (int by : {1, 2, 4, 8, 16}) {
+                if (is_stream ? (bx != 1 || by < 4) : by > 4) continue;
                 rodinia_tune_row row;
                 memset(&row, 0, sizeof row);
                 row.g = g0;

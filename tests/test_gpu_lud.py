@@ -82,8 +82,9 @@ def test_all_variants_bit_identical(rg):
         base = _lu(rg, A, panel, UNC).cpu().numpy()
         for r in rg.rodinia_variants("lud"):
             g = r["g"]
-            for bx, by in [(1, 1), (2, 1), (7, 3)]:
-                gg = (g[0], g[1], bx, by, 1, g[5], 0)
+            stream = bool(g[6] & rg.RODINIA_STREAM)
+            for bx, by in ([(1, 1), (1, 5)] if stream else [(1, 1), (2, 1), (7, 3)]):
+                gg = (g[0], g[1], bx, by, 1, g[5], g[6])
                 try:
                     got = _lu(rg, A, panel, gg).cpu().numpy()
                 except rg.RodiniaError as e:
