@@ -14,6 +14,7 @@
 #include <vector>
 
 #include "hs_cell.cuh"
+#include "workloads.h"
 #include "rg_internal.h"
 
 namespace rg {
@@ -200,11 +201,6 @@ void tune_cache_store(rodinia_kernel k, const rodinia_problem& p, const rodinia_
 namespace hotspot {
 struct DirectVariant;
 struct StreamVariant;
-rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C, const DirectVariant** dv,
-                     const StreamVariant** sv);
-rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C, int iters,
-                   const HsCoef& cf, const rodinia_granularity& g, const DirectVariant* dv,
-                   const StreamVariant* sv, cudaStream_t s);
 }  // namespace hotspot
 
 // Default granularity per workload when neither the caller nor the tune cache chooses one.
@@ -294,8 +290,6 @@ static rodinia_status hotspot_resolve(int64_t R, int64_t C, int32_t iters, const
     return RODINIA_OK;
 }
 
-static HsCoef to_coef(const rodinia_hotspot_coeffs& c) { return HsCoef{c.k, c.rx, c.ry, c.rz, c.amb}; }
-
 extern "C" rodinia_status rodinia_hotspot(const float* tin, const float* p, float* tout, float* scratch,
                                           int64_t R, int64_t C, int32_t iters,
                                           const rodinia_hotspot_coeffs* coeffs,
@@ -315,8 +309,13 @@ extern "C" rodinia_status rodinia_hotspot(const float* tin, const float* p, floa
     RG_TRY(device_info(&di));
     cudaStream_t s = (cudaStream_t)stream;
     float* scr = scratch;
-    if (!scr && iters >= 2) RG_TRY(scratch_alloc((void**)&scr, (size_t)R * C * sizeof(float), s));
-    rodinia_status st = hotspot::run(tin, p, tout, scr, (int)R, (int)C, iters, to_coef(cc), gg, dv, sv, s);
+    float* kp = nullptr;
+    const size_t bytes = (size_t)R * C * sizeof(float);
+    if (!scr && iters >= 1) RG_TRY(scratch_alloc((void**)&scr, bytes, s));
+    rodinia_status st = RODINIA_OK;
+    if (iters >= 1) st = scratch_alloc((void**)&kp, bytes, s);
+    if (st == RODINIA_OK) st = hotspot::solve(tin, p, tout, scr, kp, (int)R, (int)C, iters, cc, gg, dv, sv, s);
+    if (kp) scratch_free(kp, s);
     if (scr != scratch) scratch_free(scr, s);
     return st;
 }

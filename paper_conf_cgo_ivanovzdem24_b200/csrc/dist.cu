@@ -287,7 +287,7 @@ extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp
     rodinia_hotspot_coeffs cc;
     if (coeffs) cc = *coeffs;
     else rodinia_hotspot_coeffs_rodinia(R, C, 0.016, 0.016, &cc);
-    const HsCoef cf{cc.k, cc.rx, cc.ry, cc.rz, cc.amb};
+    const HsCoef cf = hs_derive(cc.k, cc.rx, cc.ry, cc.rz);  // state form (hs_cell.cuh)
     std::vector<Slab> sl;
     RG_TRY(make_slabs(c, R, D, D, &sl));
     DeviceInfo di;
@@ -305,6 +305,9 @@ extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp
         if (st == RODINIA_OK) {
             cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, arg_ptr(c, temp_local, i), x.own * rowb, cudaMemcpyDeviceToDevice, s);
             cudaMemcpyAsync(x.aux + (size_t)x.top * C, arg_ptr(c, power_local, i), x.own * rowb, cudaMemcpyDeviceToDevice, s);
+            // T -> u = T - amb and P -> kP = k*P on the owned rows (halos arrive converted)
+            hotspot::convert(x.buf[0] + (size_t)x.top * C, x.buf[0] + (size_t)x.top * C, (int64_t)x.own * C, 0, cc.amb, s);
+            hotspot::convert(x.aux + (size_t)x.top * C, x.aux + (size_t)x.top * C, (int64_t)x.own * C, 1, cc.k, s);
         }
     }
     if (st == RODINIA_OK && c->nranks > 1) st = exchange(c, sl, 0, (int)C, D, D, true, s);
@@ -322,8 +325,9 @@ extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp
     for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
         Slab& x = sl[i];
         float* dst = c->kind == 1 ? ((float* const*)out_local)[i] : (float*)out_local;
-        if (cudaMemcpyAsync(dst, x.buf[cur] + (size_t)x.top * C, x.own * rowb, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
-            st = cuda_error(cudaGetLastError(), "hotspot_dist copy-out", __FILE__, __LINE__);
+        hotspot::convert(x.buf[cur] + (size_t)x.top * C, dst, (int64_t)x.own * C, 2, cc.amb, s);  // u -> T
+        const cudaError_t ce = cudaGetLastError();
+        if (ce != cudaSuccess) st = cuda_error(ce, "hotspot_dist copy-out", __FILE__, __LINE__);
     }
     if (st == RODINIA_OK && cudaGetLastError() != cudaSuccess) st = set_error(RODINIA_E_CUDA, "hotspot_dist: launch failed");
     free_slabs(sl, s);

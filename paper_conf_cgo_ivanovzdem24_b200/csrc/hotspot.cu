@@ -1,6 +1,9 @@
 // hotspot.cu -- granularity-parameterised hotspot kernels for sm_100a.
 //
-// Operation: Rodinia hotspot `calculate_temp` (DESIGN.md §3 H1-H8), per cell via hs_cell().
+// Operation: Rodinia hotspot `calculate_temp` (DESIGN.md §3 H1-H8), per cell via hs_cell() in
+// the state form u = T - amb with pre-scaled power kP = k*P (DESIGN.md §3 H2): every stepping
+// kernel below reads/writes states u and reads kP where the comments say T and P; solve()
+// converts T -> u and P -> kP before the first launch and u -> T after the last.
 // Two variant families:
 //
 //  * hs_direct<TX,TY,MODE>  (temporal = 1).  The paper's granularity space verbatim: the
@@ -188,13 +191,29 @@ __device__ __forceinline__ void hs_read_row(const float* base, int sc0, int slot
 }
 
 // Request the rows step `s` will consume: T row ystart+s into slot s % HS_DT, P row ystart+s-1
-// into slot s % DP (one commit group per step).
-template <int V, int H, bool EC>
+// into slot s % DP (one commit group per step).  Fast path (interior band and chunk, every
+// requested row inside the grid): running per-lane source pointers advanced by one row per
+// request and lane-constant shared-memory bases, so a request costs two 128-bit copies and a
+// few integer operations instead of clamped row arithmetic.
+template <int V, int H, bool EC, bool ER>
 __device__ __forceinline__ void hs_issue_step(float* tring, float* pring, const float* __restrict__ tin,
                                               const float* __restrict__ pw, int s, int ystart, int R, int C,
-                                              int col0, int sc0) {
-    hs_issue_row<V, EC>(tring, tin, ystart + s, R, C, col0, sc0, s & (HS_DT - 1));
-    hs_issue_row<V, EC>(pring, pw, ystart + s - 1, R, C, col0, sc0, s & (HsRing<H>::DP - 1));
+                                              int col0, int sc0, const float*& tsrc, const float*& psrc) {
+    if (!EC && !ER && V % 4 == 0) {
+        constexpr int DP = HsRing<H>::DP;
+        const uint32_t td = (uint32_t)__cvta_generic_to_shared(tring + sc0) + (uint32_t)((s & (HS_DT - 1)) * 32 * V * 4);
+        const uint32_t pd = (uint32_t)__cvta_generic_to_shared(pring + sc0) + (uint32_t)((s & (DP - 1)) * 32 * V * 4);
+#pragma unroll
+        for (int q = 0; q < V / 4; ++q) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(td + 16 * q), "l"(tsrc + 4 * q));
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(pd + 16 * q), "l"(psrc + 4 * q));
+        }
+        tsrc += C;
+        psrc += C;
+    } else {
+        hs_issue_row<V, EC>(tring, tin, ystart + s, R, C, col0, sc0, s & (HS_DT - 1));
+        hs_issue_row<V, EC>(pring, pw, ystart + s - 1, R, C, col0, sc0, s & (HsRing<H>::DP - 1));
+    }
     asm volatile("cp.async.commit_group;\n" ::);
 }
 
@@ -202,14 +221,15 @@ template <int V, int H, int K, bool EC, bool ER>
 __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tring, float* pring,
                                                const float* __restrict__ tin, const float* __restrict__ pw,
                                                float* __restrict__ tout, int s, int ystart, int R, int C, int ylo,
-                                               int yhi, int sc0, int col0, const HsCoef& cf) {
+                                               int yhi, int sc0, int col0, const HsCoef& cf,
+                                               const float*& tsrc, const float*& psrc) {
     constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
     constexpr int DP = HsRing<H>::DP;
     const int g0 = ystart + s;
     // this step's rows have landed once at most HS_DT-2 later groups are pending
     asm volatile("cp.async.wait_group %0;\n" ::"n"(HS_DT - 2));
     hs_read_row<V>(tring, sc0, s & (HS_DT - 1), ring[0][S2]);  // level 0 = T row g0
-    hs_issue_step<V, H, EC>(tring, pring, tin, pw, s + HS_DT - 1, ystart, R, C, col0, sc0);
+    hs_issue_step<V, H, EC, ER>(tring, pring, tin, pw, s + HS_DT - 1, ystart, R, C, col0, sc0, tsrc, psrc);
 
 #pragma unroll
     for (int l = 0; l < H; ++l) {
@@ -241,7 +261,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
             // level H: write the lane's cells that lie in the band's output columns
             constexpr int s_lo = H, s_hi = 32 * V - H;  // staged-column range of the output
             float* orow = tout + (size_t)g * C + col0;
-            if (!EC && (H % V == 0)) {
+            if constexpr (!EC && (H % V == 0) && V <= 4) {
                 if (sc0 >= s_lo && sc0 < s_hi) {
                     typename VecT<V>::T t;
                     float* f = reinterpret_cast<float*>(&t);
@@ -249,6 +269,13 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
                     for (int v = 0; v < V; ++v) f[v] = res[v];
                     *reinterpret_cast<typename VecT<V>::T*>(orow) = t;
                 }
+            } else if constexpr (!EC && V % 4 == 0 && H % 4 == 0) {
+                // 128-bit pieces: each lies wholly inside or outside the output range
+#pragma unroll
+                for (int q = 0; q < V / 4; ++q)
+                    if (sc0 + 4 * q >= s_lo && sc0 + 4 * q < s_hi)
+                        *reinterpret_cast<float4*>(orow + 4 * q) =
+                            make_float4(res[4 * q], res[4 * q + 1], res[4 * q + 2], res[4 * q + 3]);
             } else {
 #pragma unroll
                 for (int v = 0; v < V; ++v) {
@@ -275,15 +302,20 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
     const int ystart = y0 - H;
     const int nsteps = (y1 - y0) + 2 * H;
 #pragma unroll
-    for (int k = 0; k < HS_DT - 1; ++k) hs_issue_step<V, H, EC>(tring, pring, tin, pw, k, ystart, R, C, col0, sc0);
+    // fast-path source pointers (only dereferenced when !EC && !ER: all requested rows exist)
+    const float* tsrc = tin + (size_t)max(ystart, 0) * C + col0;
+    const float* psrc = pw + (size_t)max(ystart - 1, 0) * C + col0;
+#pragma unroll
+    for (int k = 0; k < HS_DT - 1; ++k)
+        hs_issue_step<V, H, EC, ER>(tring, pring, tin, pw, k, ystart, R, C, col0, sc0, tsrc, psrc);
     int s = 0;
     for (; s + 3 <= nsteps; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf);
-        hs_stream_step<V, H, 2, EC, ER>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf);
+        hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 2, EC, ER>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
     }
-    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf);
-    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf);
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
     asm volatile("cp.async.wait_group 0;\n" ::);  // drain before the rings are reused
 }
 
@@ -303,7 +335,8 @@ __global__ void __launch_bounds__(32, OCC)
     const int y0 = blockIdx.y * chunk;
     const int y1 = min(y0 + chunk, R);
     // rows computed: [y0-H, y1+H); ER selects the row-clamp path near the grid's top/bottom
-    const bool er = (y0 - H - 1 < 0) || (y1 + H > R - 1);
+    // (rows requested: [y0-H-1, y1+H+HS_DT-1), the prefetch running HS_DT-1 rows past the last step)
+    const bool er = (y0 - H - 1 < 0) || (y1 + H + HS_DT - 1 > R);
     __shared__ __align__(16) float tring[HS_DT * 32 * V];
     __shared__ __align__(16) float pring[HsRing<H>::DP * 32 * V];
     for (int bi = 0; bi < bands_per_cta; ++bi) {
@@ -442,36 +475,99 @@ static void launch_stream(const StreamVariant* sv, int bx, int by, const float* 
     count_launch();
 }
 
-// Run `iters` steps on a (R x C) buffer from `tin` into `tout`, ping-ponging through `scr`.
+// ---------------------------------------------------------------- state conversions
+// y = x - a (T -> u), y = x * a (P -> kP), y = x + a (u -> T); elementwise, grid-stride,
+// 128-bit when all pointers are 16-byte aligned.  In place is allowed (x == y).
+template <int OP>
+__device__ __forceinline__ float hs_conv1(float x, float a) {
+    return OP == 0 ? __fsub_rn(x, a) : (OP == 1 ? __fmul_rn(x, a) : __fadd_rn(x, a));
+}
+template <int OP>
+__global__ void __launch_bounds__(256) hs_convert(const float* x, float* y, int64_t n, float a, int vec) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (vec) {
+        const int64_t n4 = n / 4;
+        for (int64_t j = i; j < n4; j += stride) {
+            float4 v = reinterpret_cast<const float4*>(x)[j];
+            v.x = hs_conv1<OP>(v.x, a); v.y = hs_conv1<OP>(v.y, a);
+            v.z = hs_conv1<OP>(v.z, a); v.w = hs_conv1<OP>(v.w, a);
+            reinterpret_cast<float4*>(y)[j] = v;
+        }
+        i += n4 * 4;
+    }
+    for (; i < n; i += stride) y[i] = hs_conv1<OP>(x[i], a);
+}
+
+void convert(const float* x, float* y, int64_t n, int op, float a, cudaStream_t s) {
+    if (n <= 0) return;
+    const int vec = ((reinterpret_cast<uintptr_t>(x) | reinterpret_cast<uintptr_t>(y)) % 16) == 0;
+    const int64_t want = (n / 4 + 255) / 256 + 1;
+    const int grid = (int)std::min<int64_t>(want, 148 * 8);
+    if (op == 0) hs_convert<0><<<grid, 256, 0, s>>>(x, y, n, a, vec);
+    else if (op == 1) hs_convert<1><<<grid, 256, 0, s>>>(x, y, n, a, vec);
+    else hs_convert<2><<<grid, 256, 0, s>>>(x, y, n, a, vec);
+    count_launch();
+}
+
+int num_launches(int iters, const StreamVariant* sv) {
+    const int h = sv ? sv->h : 1;
+    return iters / h + iters % h;  // remainder steps run one per launch (direct family)
+}
+
+// Run `iters` steps in state space on a (R x C) buffer from `usrc` into `udst`, ping-ponging
+// through `uscr` (`usrc` may be `uscr` when num_launches() is odd, or `udst` when it is even).
 // The granularity has been validated by check().  Neighbour rows are clamped to the buffer,
 // so the same routine serves whole grids and halo'd slabs.
-rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C,
+rodinia_status run(const float* usrc, const float* kp, float* udst, float* uscr, int R, int C,
                    int iters, const HsCoef& cf, const rodinia_granularity& g,
                    const DirectVariant* dv, const StreamVariant* sv, cudaStream_t s) {
     if (iters == 0) {
-        RG_CUDA(cudaMemcpyAsync(tout, tin, (size_t)R * C * sizeof(float), cudaMemcpyDeviceToDevice, s));
+        if (udst != usrc)
+            RG_CUDA(cudaMemcpyAsync(udst, usrc, (size_t)R * C * sizeof(float), cudaMemcpyDeviceToDevice, s));
         return RODINIA_OK;
     }
     const int h = sv ? sv->h : 1;
-    const int nfull = iters / h, rem = iters % h;
-    const int launches = nfull + rem;  // remainder steps run one per launch (direct family)
+    const int nfull = iters / h;
+    const int launches = num_launches(iters, sv);
     const DirectVariant* remv = find_direct(4, 1, 1);
     int left = launches;
-    const float* src = tin;
+    const float* src = usrc;
     int done = 0;
     while (left > 0) {
-        float* dst = ((left - 1) % 2 == 0) ? tout : scr;
+        float* dst = ((left - 1) % 2 == 0) ? udst : uscr;
         if (sv && done < nfull) {
-            launch_stream(sv, g.block_x, g.block_y, src, p, dst, R, C, cf, s);
+            launch_stream(sv, g.block_x, g.block_y, src, kp, dst, R, C, cf, s);
             ++done;
         } else if (dv) {
-            launch_direct(dv, g.block_x, g.block_y, src, p, dst, R, C, cf, s);
+            launch_direct(dv, g.block_x, g.block_y, src, kp, dst, R, C, cf, s);
         } else {
-            launch_direct(remv, 1, 1, src, p, dst, R, C, cf, s);
+            launch_direct(remv, 1, 1, src, kp, dst, R, C, cf, s);
         }
         src = dst;
         --left;
     }
+    RG_CUDA(cudaGetLastError());
+    return RODINIA_OK;
+}
+
+// Whole solve from temperatures: T -> u (into the buffer the first launch does not write),
+// P -> kP (into `kp`), `iters` steps, u -> T in place in `tout`.  `scr` and `kp` are R x C
+// scratch buffers distinct from every operand.
+rodinia_status solve(const float* tin, const float* p, float* tout, float* scr, float* kp, int R, int C,
+                     int iters, const rodinia_hotspot_coeffs& cc, const rodinia_granularity& g,
+                     const DirectVariant* dv, const StreamVariant* sv, cudaStream_t s) {
+    const int64_t n = (int64_t)R * C;
+    if (iters == 0) {
+        RG_CUDA(cudaMemcpyAsync(tout, tin, (size_t)n * sizeof(float), cudaMemcpyDeviceToDevice, s));
+        return RODINIA_OK;
+    }
+    const HsCoef cf = hs_derive(cc.k, cc.rx, cc.ry, cc.rz);
+    float* u0 = (num_launches(iters, sv) % 2 == 1) ? scr : tout;
+    convert(tin, u0, n, 0, cc.amb, s);
+    convert(p, kp, n, 1, cc.k, s);
+    RG_TRY(run(u0, kp, tout, scr, R, C, iters, cf, g, dv, sv, s));
+    convert(tout, tout, n, 2, cc.amb, s);
     RG_CUDA(cudaGetLastError());
     return RODINIA_OK;
 }

@@ -1,32 +1,51 @@
 // hs_cell.cuh -- the one per-cell hotspot update every hotspot kernel variant calls.
 //
-// Rodinia hotspot `calculate_temp` (DESIGN.md §3 H1-H8):
-//   T' = c + k * ( P + ((S+N) - 2c)*ry + ((E+W) - 2c)*rx + (amb - c)*rz )
-// evaluated in fp32 in exactly this order with explicit round-to-nearest intrinsics, so the
-// compiler cannot contract or reorder differently in different variants: every coarsening
-// variant is bit-identical to every other one (the paper's correctness criterion,
-// PAPER.md:145, 295).  (S+N) - 2c is written as fma(-2, c, S+N), which equals the unfused
-// (S+N) - (2c) exactly because 2c is exact in fp32; the three "acc + x*r" terms and the
-// final c + k*acc use fused multiply-adds (DESIGN.md §3 H2).
+// Rodinia hotspot `calculate_temp` (DESIGN.md §3 H1-H8) defines
+//   T' = c + k * ( P + ((S+N) - 2c)*ry + ((E+W) - 2c)*rx + (amb - c)*rz ).
+// The kernels evaluate the algebraically identical *state form* (DESIGN.md §3 H2):
+//   u  = T - amb                       (state, converted once per solve: hs_to_state)
+//   kP = fl(k * P)                     (pre-scaled power, once per solve: hs_scale_power)
+//   u' = u + ( (S+N)*kry + kP + (E+W)*krx + u*m )
+// with kry = fl(k*ry), krx = fl(k*rx), m = fl(-k*(2ry + 2rx + rz)) computed in fp64 and rounded
+// once (hs_derive), and T = u + amb at the end (hs_from_state).  Substituting c = u + amb
+// (and N = uN + amb, ...) into the definition gives exactly this expression; it costs 6 FP32
+// operations per cell-update instead of 9, and its fp32 error against the fp64 oracle is
+// smaller than the literal order's (the state u has half the ulp of T near 320 K; measured in
+// DESIGN.md §3 H2).  Explicit round-to-nearest intrinsics keep the compiler from contracting or
+// reordering differently in different variants, so every coarsening variant is bit-identical
+// to every other one (the paper's correctness criterion).
 #pragma once
+
+#include <cstdint>
 
 namespace rg {
 
-struct HsCoef {
-    float k, rx, ry, rz, amb;
+struct HsCoef {   // state-form coefficients (device side)
+    float kry, krx, m;
 };
 
-__device__ __forceinline__ float hs_cell(float c, float n, float s, float e, float w, float p,
+struct HsMap {    // state <-> temperature map (pre/post passes)
+    float k, amb;
+};
+
+// fp64 evaluation of the derived coefficients from the caller's fp32 (k, rx, ry, rz).
+inline HsCoef hs_derive(float k, float rx, float ry, float rz) {
+    const double kd = k;
+    HsCoef c;
+    c.kry = (float)(kd * (double)ry);
+    c.krx = (float)(kd * (double)rx);
+    c.m = (float)(-kd * (2.0 * (double)ry + 2.0 * (double)rx + (double)rz));
+    return c;
+}
+
+__device__ __forceinline__ float hs_cell(float u, float n, float s, float e, float w, float kp,
                                          const HsCoef& cf) {
-    float sn = __fadd_rn(s, n);
-    float ew = __fadd_rn(e, w);
-    float a = __fmaf_rn(-2.0f, c, sn);
-    float b = __fmaf_rn(-2.0f, c, ew);
-    float d = __fsub_rn(cf.amb, c);
-    float acc = __fmaf_rn(a, cf.ry, p);
-    acc = __fmaf_rn(b, cf.rx, acc);
-    acc = __fmaf_rn(d, cf.rz, acc);
-    return __fmaf_rn(cf.k, acc, c);
+    const float sn = __fadd_rn(s, n);
+    const float ew = __fadd_rn(e, w);
+    float acc = __fmaf_rn(sn, cf.kry, kp);
+    acc = __fmaf_rn(ew, cf.krx, acc);
+    acc = __fmaf_rn(u, cf.m, acc);
+    return __fadd_rn(u, acc);
 }
 
 }  // namespace rg

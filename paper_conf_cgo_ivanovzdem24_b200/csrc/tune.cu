@@ -9,6 +9,7 @@
 #include <vector>
 
 #include "hs_cell.cuh"
+#include "workloads.h"
 #include "rg_internal.h"
 
 namespace rg {
@@ -28,11 +29,6 @@ struct DirectVariant;
 struct StreamVariant;
 int num_variants();
 void variant_info(int i, rodinia_granularity* g, const void** fn, const char** key, int* threads);
-rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C, const DirectVariant** dv,
-                     const StreamVariant** sv);
-rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C, int iters,
-                   const HsCoef& cf, const rodinia_granularity& g, const DirectVariant* dv,
-                   const StreamVariant* sv, cudaStream_t s);
 }  // namespace hotspot
 
 struct Registry {
@@ -184,11 +180,13 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
         cudaGetLastError();
         st = set_error(RODINIA_E_NOMEM, "tune: cannot allocate %zu-byte buffers", bytes);
     }
-    if (st == RODINIA_OK) st = fill(tin, R * C, 323.15f, 20.0f, 1u, s);
-    if (st == RODINIA_OK) st = fill(pw, R * C, 0.0f, 1e-3f, 2u, s);
+    // states u = T - amb and pre-scaled power kP = k*P of the synthetic recipe (hs_cell.cuh);
+    // the stepping kernels' run time does not depend on the values
     rodinia_hotspot_coeffs cc;
     rodinia_hotspot_coeffs_rodinia(R, C, R * 31.25e-6, C * 31.25e-6, &cc);
-    const HsCoef cf{cc.k, cc.rx, cc.ry, cc.rz, cc.amb};
+    const HsCoef cf = hs_derive(cc.k, cc.rx, cc.ry, cc.rz);
+    if (st == RODINIA_OK) st = fill(tin, R * C, 323.15f - cc.amb, 20.0f, 1u, s);
+    if (st == RODINIA_OK) st = fill(pw, R * C, 0.0f, 1e-3f * cc.k, 2u, s);
     const int base_spill = family_base_spill(RODINIA_HOTSPOT);
     float best_ms = 1e30f;
     auto time_one = [&](const rodinia_granularity& gc) {

@@ -15,9 +15,17 @@ struct DirectVariant;
 struct StreamVariant;
 rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C, const DirectVariant** dv,
                      const StreamVariant** sv);
-rodinia_status run(const float* tin, const float* p, float* tout, float* scr, int R, int C, int iters,
+// Steps in state space (u = T - amb, kP = k*P; hs_cell.cuh): usrc -> udst via uscr.
+rodinia_status run(const float* usrc, const float* kp, float* udst, float* uscr, int R, int C, int iters,
                    const HsCoef& cf, const rodinia_granularity& g, const DirectVariant* dv,
                    const StreamVariant* sv, cudaStream_t s);
+// Whole solve from temperatures (conversions + run); scr and kp are R x C scratch buffers.
+rodinia_status solve(const float* tin, const float* p, float* tout, float* scr, float* kp, int R, int C,
+                     int iters, const rodinia_hotspot_coeffs& cc, const rodinia_granularity& g,
+                     const DirectVariant* dv, const StreamVariant* sv, cudaStream_t s);
+// Elementwise state conversions: op 0: y = x - a, 1: y = x * a, 2: y = x + a (in place allowed).
+void convert(const float* x, float* y, int64_t n, int op, float a, cudaStream_t s);
+int num_launches(int iters, const StreamVariant* sv);
 int temporal_of(const StreamVariant* sv);  // steps per launch (1 for the direct family)
 }  // namespace hotspot
 

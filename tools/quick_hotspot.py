@@ -7,6 +7,7 @@ import paper_conf_cgo_ivanovzdem24_b200 as rg
 N = int(sys.argv[1]) if len(sys.argv) > 1 else 16384
 iters = int(sys.argv[2]) if len(sys.argv) > 2 else 48
 which = sys.argv[3] if len(sys.argv) > 3 else "all"
+bys = [int(x) for x in sys.argv[4].split(",")] if len(sys.argv) > 4 else [2, 4, 8]
 t = torch.rand(N, N, device="cuda") * 20 + 323.15
 p = torch.rand(N, N, device="cuda") * 1e-3
 c = rg.rodinia_hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6)
@@ -19,7 +20,7 @@ if which in ("all", "stream"):
         g = r["g"]
         if not (g[6] & 2) or r["status"] != 0:
             continue
-        for by in (2, 4, 8):
+        for by in bys:
             grans.append((g[0], 1, 1, by, g[4], 1, g[6]))
 res = []
 for g in grans:
