@@ -240,11 +240,10 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
         const float wnb = __shfl_up_sync(0xffffffffu, ring[l][S1][V - 1], 1);
         const float enb = __shfl_down_sync(0xffffffffu, ring[l][S1][0], 1);
         float res[V];
+        float ew[V];
 #pragma unroll
         for (int v = 0; v < V; ++v) {
             const float c = ring[l][S1][v];
-            const float n = top ? c : ring[l][S0][v];
-            const float s_ = bot ? c : ring[l][S2][v];
             float w = v > 0 ? ring[l][S1][v > 0 ? v - 1 : 0] : wnb;
             float e = v < V - 1 ? ring[l][S1][v < V - 1 ? v + 1 : 0] : enb;
             if (EC) {
@@ -252,7 +251,29 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
                 if (col == 0) w = c;
                 if (col == C - 1) e = c;
             }
-            res[v] = hs_cell(c, n, s_, e, w, pv[v], cf);
+            ew[v] = __fadd_rn(e, w);
+        }
+        if constexpr (V % 2 == 0) {
+            // column pairs through the packed FP32x2 pipe (FADD2/FFMA2): same per-element
+            // operations and roundings as hs_cell, half the issue slots (hs_cell2)
+#pragma unroll
+            for (int q = 0; q < V / 2; ++q) {
+                const int v0 = 2 * q, v1 = 2 * q + 1;
+                const float2 c2 = make_float2(ring[l][S1][v0], ring[l][S1][v1]);
+                const float2 n2 = top ? c2 : make_float2(ring[l][S0][v0], ring[l][S0][v1]);
+                const float2 s2 = bot ? c2 : make_float2(ring[l][S2][v0], ring[l][S2][v1]);
+                const float2 r = hs_cell2(c2, n2, s2, make_float2(ew[v0], ew[v1]), make_float2(pv[v0], pv[v1]), cf);
+                res[v0] = r.x;
+                res[v1] = r.y;
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+                const float c = ring[l][S1][v];
+                const float n = top ? c : ring[l][S0][v];
+                const float s_ = bot ? c : ring[l][S2][v];
+                res[v] = hs_cell_ew(c, n, s_, ew[v], pv[v], cf);
+            }
         }
         if (l + 1 < H) {
 #pragma unroll

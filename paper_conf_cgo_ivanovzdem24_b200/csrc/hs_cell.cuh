@@ -38,6 +38,26 @@ inline HsCoef hs_derive(float k, float rx, float ry, float rz) {
     return c;
 }
 
+// The same update with E+W already formed (ew = fl(e + w)).
+__device__ __forceinline__ float hs_cell_ew(float u, float n, float s, float ew, float kp, const HsCoef& cf) {
+    const float sn = __fadd_rn(s, n);
+    float acc = __fmaf_rn(sn, cf.kry, kp);
+    acc = __fmaf_rn(ew, cf.krx, acc);
+    acc = __fmaf_rn(u, cf.m, acc);
+    return __fadd_rn(u, acc);
+}
+
+// Two cells at once on the packed FP32x2 pipe (sm_100 FADD2/FFMA2): element-wise the same
+// operations in the same order with the same round-to-nearest as hs_cell_ew, so the results
+// are bit-identical; one instruction covers both cells.
+__device__ __forceinline__ float2 hs_cell2(float2 u, float2 n, float2 s, float2 ew, float2 kp, const HsCoef& cf) {
+    const float2 sn = __fadd2_rn(s, n);
+    float2 acc = __ffma2_rn(sn, make_float2(cf.kry, cf.kry), kp);
+    acc = __ffma2_rn(ew, make_float2(cf.krx, cf.krx), acc);
+    acc = __ffma2_rn(u, make_float2(cf.m, cf.m), acc);
+    return __fadd2_rn(u, acc);
+}
+
 __device__ __forceinline__ float hs_cell(float u, float n, float s, float e, float w, float kp,
                                          const HsCoef& cf) {
     const float sn = __fadd_rn(s, n);

@@ -146,7 +146,7 @@ static void hotspot_stage2(const rodinia_granularity& base, std::vector<rodinia_
     rodinia_granularity g = base;
     if (g.flags & RODINIA_STREAM) {
         for (int bx : {1, 2})
-            for (int by : {2, 3, 4, 6, 8, 16}) { g.block_x = bx; g.block_y = by; out->push_back(g); }
+            for (int by : {2, 3, 4, 6, 8, 12, 16, 24}) { g.block_x = bx; g.block_y = by; out->push_back(g); }
     } else {
         static const int bxy[][2] = {{1, 1}, {2, 1}, {3, 1}, {4, 1}, {7, 1}, {1, 2}, {2, 2}, {4, 4}};
         for (auto& b : bxy) { g.block_x = b[0]; g.block_y = b[1]; out->push_back(g); }
