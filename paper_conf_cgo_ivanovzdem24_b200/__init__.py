@@ -15,7 +15,7 @@ import os
 from dataclasses import dataclass
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "librodinia_gran.so")
+LIB_PATH = os.environ.get("RODINIA_GRAN_LIB") or os.path.join(_HERE, "librodinia_gran.so")  # env: dev A/B builds
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

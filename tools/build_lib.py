@@ -38,7 +38,7 @@ def _newest(paths):
     return max((os.path.getmtime(p) for p in paths), default=0.0)
 
 
-def _compile(src: str, force: bool) -> tuple[str, str]:
+def _compile(src: str, force: bool, extra=()) -> tuple[str, str]:
     name = os.path.splitext(os.path.basename(src))[0]
     obj = os.path.join(BUILD, name + ".o")
     log = os.path.join(BUILD, f"ptxas_{name}.log")
@@ -46,7 +46,7 @@ def _compile(src: str, force: bool) -> tuple[str, str]:
         [os.path.join(ROOT, "include", "rodinia_gran.h")]
     if not force and os.path.exists(obj) and os.path.exists(log) and os.path.getmtime(obj) >= _newest(deps):
         return obj, log
-    cmd = [NVCC, *CFLAGS, "-c", src, "-o", obj]
+    cmd = [NVCC, *CFLAGS, *extra, "-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
@@ -55,11 +55,20 @@ def _compile(src: str, force: bool) -> tuple[str, str]:
     return obj, log
 
 
-def build(force: bool = False, jobs: int = 8, verbose: bool = True) -> str:
+def build(force: bool = False, jobs: int = 8, verbose: bool = True, defines=(), out: str = "",
+          builddir: str = "") -> str:
+    """defines/out/builddir: development A/B builds (e.g. -D RG_SR_D=8 into a second .so that
+    the binding loads when RODINIA_GRAN_LIB names it); the default build uses none of them."""
+    global BUILD, LIB
+    if builddir:
+        BUILD = os.path.abspath(builddir)
+    if out:
+        LIB = os.path.abspath(out)
     os.makedirs(BUILD, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    extra = [f"-D{d}" for d in defines]
     with cf.ThreadPoolExecutor(max_workers=jobs) as ex:
-        results = list(ex.map(lambda s: _compile(s, force), srcs))
+        results = list(ex.map(lambda s: _compile(s, force, extra), srcs))
     objs = [o for o, _ in results]
     text = "".join(open(l).read() for _, l in results)
     stats = ptxas_filter.parse_ptxas_log(text)
@@ -89,5 +98,8 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("-j", type=int, default=8)
+    ap.add_argument("--define", action="append", default=[])
+    ap.add_argument("--out", default="")
+    ap.add_argument("--builddir", default="")
     a = ap.parse_args()
-    build(force=a.force, jobs=a.j)
+    build(force=a.force, jobs=a.j, defines=a.define, out=a.out, builddir=a.builddir)

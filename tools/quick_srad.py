@@ -12,7 +12,7 @@ J = J0.clone()
 grans = [(1,1,1,1,1,0,0), (2,1,4,2,1,0,0), (2,1,4,2,1,1,0)]
 for v in (1, 2, 4, 8):
     for bx in (1, 2):
-        for by in (2, 4, 8, 16, 32):
+        for by in (1, 2, 3, 4, 8):
             grans.append((v, 1, bx, by, 1, 1, 2))
 res = []
 for g in grans:
