@@ -175,11 +175,13 @@ def run_reference(args):
 
 
 # ----------------------------------------------------------------------------- GPU arm
-def _time_steps(fn, steps, warmup, stream):
+def _time_steps(fn, steps, warmup, stream, on_start=None):
     import torch
     for _ in range(warmup):
         fn()
     torch.cuda.synchronize()
+    if on_start:
+        on_start()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     e0.record(stream)
@@ -432,21 +434,25 @@ def run_ours(args):
     torch.cuda.synchronize()
     l0 = rg.rodinia_launch_count()
     with ClockSampler(local) as clk:
-        ms = _time_steps(step, args.steps, args.warmup, stream)
+        ms = _time_steps(step, args.steps, args.warmup, stream, on_start=lambda: rg.rodinia_kernel_timing(True))
+    k_ms, k_launches = rg.rodinia_kernel_time()  # event pairs around every stepping launch
+    rg.rodinia_kernel_timing(False)
     launches_total = rg.rodinia_launch_count() - l0
     launches_timed = launches_total * args.steps // (args.steps + args.warmup)
     ms = _max_over_ranks(ms, ws)
     _barrier(ws)
     value = N * N * iters / (ms * 1e-3)
 
-    # ---- roofline of the dominant kernel (one kernel type per step, no remainder launches
-    # when iters % temporal == 0): avg launch duration = step time / launches per step.
+    # ---- roofline of the dominant kernel: its average launch duration from CUDA events the
+    # library records around each stepping launch on the bench stream inside the timed region
+    # (rodinia_kernel_timing); the state conversions (3 elementwise passes per solve) are not
+    # part of it.  Steps per launch h: all launches are full-depth when iters % h == 0.
     h = g.temporal if g.temporal >= 1 else 1
-    launches_per_step = launches_timed / args.steps
     rows_local = N if ws == 1 else N // ws
     hbm_peak, peak_src = _peaks()
     bytes_per_launch = 12.0 * rows_local * N  # algorithmic: read T, read P, write T'
-    avg_launch_ms = ms / max(launches_per_step, 1)
+    avg_launch_ms = k_ms / max(k_launches, 1)
+    avg_launch_ms = _max_over_ranks(avg_launch_ms, ws)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
     traffic = None
     # DRAM traffic per launch from the committed ncu --set full capture of the same kernel and
@@ -466,13 +472,17 @@ def run_ours(args):
             "kernel": "hs_stream" if g.flags & rg.RODINIA_STREAM else "hs_direct",
             "bytes_per_launch": bytes_per_launch, "avg_launch_ms": avg_launch_ms,
             "updates_per_launch": rows_local * N * h}
-    # The same kernel against the FP32 SIMT roof: hs_cell is 3 FADD + 6 FFMA =
-    # 15 flop per cell-update; peak = 148 SMs x 128 lanes x 2 flop x 1.965 GHz = 74.4 TFLOP/s.
-    # With H steps per launch the kernel sits near the ridge, so both fractions are reported.
+    # The same kernel against the FP32 SIMT roof: the state-form update
+    # (hs_cell.cuh) is 2 FADD + 3 FFMA + 1 FADD = 9 flop per cell-update (6 FP32 lane
+    # operations, issued as FADD2/FFMA2 pairs).  Peak = 148 SMs x 128 lanes x 2 flop x 1.965 GHz
+    # = 74.4 TFLOP/s; for this 50 % FMA mix the FP32 pipe tops out at 1.5 flop per lane-op,
+    # 55.8 TFLOP/s (= 6.2e12 cell-updates/s), reported as pipe_peak / pipe_frac.
     fp32_peak = 148 * 128 * 2 * 1.965e9 / 1e12
-    ach_tf = 15.0 * rows_local * N * h / (avg_launch_ms * 1e-3) / 1e12
+    mix_peak = 148 * 128 * 1.5 * 1.965e9 / 1e12
+    ach_tf = 9.0 * rows_local * N * h / (avg_launch_ms * 1e-3) / 1e12
     roof_alu = {"bound": "alu", "achieved": ach_tf, "peak": fp32_peak, "unit": "TFLOP/s",
-                "frac": ach_tf / fp32_peak, "flop_per_update": 15,
+                "frac": ach_tf / fp32_peak, "flop_per_update": 9, "pipe_peak": mix_peak,
+                "pipe_frac": ach_tf / mix_peak,
                 "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 x 1965 MHz"}
 
     # ---- uncoarsened variant (same timed protocol, fewer steps)

@@ -292,6 +292,13 @@ rodinia_status rodinia_sync(void* stream);          /* stream sync + sticky asyn
 int32_t rodinia_abi_version(void);
 /* Number of kernel launches this library has issued since load (for bench accounting). */
 int64_t rodinia_launch_count(void);
+/* Dominant-kernel timing (bench roofline).  enable != 0 starts recording a CUDA
+ * event pair around every stepping launch of hotspot (hs_stream / hs_direct) on the caller's
+ * stream and clears earlier records; enable == 0 stops.  rodinia_kernel_time() synchronises on
+ * the recorded events and returns the summed elapsed milliseconds and the number of timed
+ * launches since the last enable.  Host-only bookkeeping; errors: RODINIA_E_CUDA. */
+rodinia_status rodinia_kernel_timing(int32_t enable);
+rodinia_status rodinia_kernel_time(double* total_ms, int64_t* launches);
 
 #ifdef __cplusplus
 }

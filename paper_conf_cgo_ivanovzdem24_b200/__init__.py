@@ -112,6 +112,8 @@ _SIGS = {
     "rodinia_sync": ([_vp], _i32),
     "rodinia_abi_version": ([], _i32),
     "rodinia_launch_count": ([], _i64),
+    "rodinia_kernel_timing": ([_i32], _i32),
+    "rodinia_kernel_time": ([ctypes.POINTER(_f64), ctypes.POINTER(_i64)], _i32),
     "rodinia_hotspot_coeffs_rodinia": ([_i64, _i64, _f64, _f64, _PC], _i32),
     "rodinia_hotspot": ([_vp, _vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
     "rodinia_hotspot_host": ([_vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
@@ -405,6 +407,18 @@ def rodinia_sync(stream=None):
 
 def rodinia_launch_count() -> int:
     return int(lib.rodinia_launch_count())
+
+
+def rodinia_kernel_timing(enable: bool) -> None:
+    """Start (clearing earlier records) or stop event timing of the stepping launches."""
+    check(lib.rodinia_kernel_timing(1 if enable else 0), "rodinia_kernel_timing")
+
+
+def rodinia_kernel_time():
+    """(summed milliseconds, number of timed launches) since the last enable."""
+    ms, n = _f64(0.0), _i64(0)
+    check(lib.rodinia_kernel_time(ctypes.byref(ms), ctypes.byref(n)), "rodinia_kernel_time")
+    return float(ms.value), int(n.value)
 
 
 # ----------------------------------------------------------------------------- multi-GPU

@@ -233,6 +233,69 @@ extern "C" const char* rodinia_status_string(rodinia_status s) {
 extern "C" int32_t rodinia_abi_version(void) { return RODINIA_ABI_VERSION; }
 extern "C" int64_t rodinia_launch_count(void) { return g_launches.load(); }
 
+// ---------------------------------------------------------------- dominant-kernel timing
+namespace rg {
+struct KTimer {
+    std::mutex mu;
+    bool on = false;
+    std::vector<cudaEvent_t> pool;  // 2 per timed launch, reused across enables
+    size_t used = 0;
+};
+static KTimer& ktimer() {
+    static KTimer k;
+    return k;
+}
+static cudaEvent_t ktime_event() {
+    KTimer& k = ktimer();
+    if (k.used == k.pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        k.pool.push_back(e);
+    }
+    return k.pool[k.used++];
+}
+void ktime_begin(cudaStream_t s) {
+    KTimer& k = ktimer();
+    std::lock_guard<std::mutex> lk(k.mu);
+    if (!k.on) return;
+    if (k.used % 2 == 1) return;  // unmatched begin: ignore
+    cudaEvent_t e = ktime_event();
+    if (e) cudaEventRecord(e, s);
+}
+void ktime_end(cudaStream_t s) {
+    KTimer& k = ktimer();
+    std::lock_guard<std::mutex> lk(k.mu);
+    if (!k.on || k.used % 2 == 0) return;
+    cudaEvent_t e = ktime_event();
+    if (e) cudaEventRecord(e, s);
+}
+}  // namespace rg
+
+extern "C" rodinia_status rodinia_kernel_timing(int32_t enable) {
+    KTimer& k = ktimer();
+    std::lock_guard<std::mutex> lk(k.mu);
+    k.on = enable != 0;
+    if (k.on) k.used = 0;
+    return RODINIA_OK;
+}
+
+extern "C" rodinia_status rodinia_kernel_time(double* total_ms, int64_t* launches) {
+    if (!total_ms || !launches) return set_error(RODINIA_E_INVALID, "kernel_time: null argument");
+    KTimer& k = ktimer();
+    std::lock_guard<std::mutex> lk(k.mu);
+    double t = 0.0;
+    const size_t n = k.used / 2;
+    for (size_t i = 0; i < n; ++i) {
+        RG_CUDA(cudaEventSynchronize(k.pool[2 * i + 1]));
+        float ms = 0.f;
+        RG_CUDA(cudaEventElapsedTime(&ms, k.pool[2 * i], k.pool[2 * i + 1]));
+        t += ms;
+    }
+    *total_ms = t;
+    *launches = (int64_t)n;
+    return RODINIA_OK;
+}
+
 namespace rg { namespace srad { rodinia_status take_sticky(); } }
 
 extern "C" rodinia_status rodinia_sync(void* stream) {

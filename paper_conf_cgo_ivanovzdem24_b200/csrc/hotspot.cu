@@ -558,10 +558,14 @@ rodinia_status run(const float* usrc, const float* kp, float* udst, float* uscr,
     while (left > 0) {
         float* dst = ((left - 1) % 2 == 0) ? udst : uscr;
         if (sv && done < nfull) {
+            ktime_begin(s);
             launch_stream(sv, g.block_x, g.block_y, src, kp, dst, R, C, cf, s);
+            ktime_end(s);
             ++done;
         } else if (dv) {
+            ktime_begin(s);
             launch_direct(dv, g.block_x, g.block_y, src, kp, dst, R, C, cf, s);
+            ktime_end(s);
         } else {
             launch_direct(remv, 1, 1, src, kp, dst, R, C, cf, s);
         }

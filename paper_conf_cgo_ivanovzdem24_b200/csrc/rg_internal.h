@@ -31,6 +31,9 @@ void clear_error();
 
 extern std::atomic<int64_t> g_launches;
 inline void count_launch(int64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+// Dominant-kernel timing (rodinia_kernel_timing): event pair around a stepping launch.
+void ktime_begin(cudaStream_t s);
+void ktime_end(cudaStream_t s);
 
 // ------------------------------------------------------------------ device
 struct DeviceInfo {

@@ -1,13 +1,16 @@
 #!/bin/bash
-# One GPU session: bench (tuned), then the ncu launch list and a --set full capture of the
-# dominant kernel with the bench's tuned granularity.  Outputs under gpurun_out/.
+# One GPU session: bench (tuned), then the ncu launch list of the bench command and --set full
+# captures of the dominant hotspot kernel (bench granularity) and of srad_stream.  Outputs under
+# gpurun_out/; tools/ncu_summary.py turns them into profiles/ summaries.
 set -x
 TAG=${1:-r01}
 python bench.py > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
 G=$(python -c "import json;print(','.join(map(str,json.load(open('gpurun_out/bench_${TAG}.json'))['config']['granularity'])))")
 echo "tuned granularity: $G"
-ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file gpurun_out/launches_${TAG}.csv \
+ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_${TAG}.csv \
     python bench.py --steps 1 --warmup 3 --gran $G --no-extra --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:hs_ -s 12 -c 1 -o gpurun_out/prof_${TAG}_hotspot \
+ncu --set full --clock-control none --import-source on -k regex:hs_stream -s 12 -c 1 -o gpurun_out/prof_${TAG}_hotspot \
     python bench.py --steps 1 --warmup 3 --gran $G --no-extra --no-cpu --iters 48 > gpurun_out/ncu_${TAG}.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:srad_stream -s 3 -c 1 -o gpurun_out/prof_${TAG}_srad \
+    python tools/_srad_profile.py > gpurun_out/ncu_${TAG}_srad.log 2>&1
 tail -2 gpurun_out/ncu_${TAG}.log
