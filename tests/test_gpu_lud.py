@@ -116,3 +116,43 @@ def test_host_entry(rg):
     got = rg.rodinia_lud_host(A, 16, g=(2, 1, 2, 1, 1, 1, 0))
     L, U = oracle.lud_unpack(got.astype(np.float64))
     assert np.abs(L @ U - A).max() / np.abs(A).max() <= 1e-5
+
+
+# ---------------------------------------------------------------- panel 128: tensor cores
+# Two-level blocking with the rank-128 trailing update on tcgen05 (kind::tf32, 3xTF32 split;
+# DESIGN.md §5).  Same parity criteria (L3); integer factors stay bit-exact because every
+# operand is exactly a TF32 value (lo parts are 0) and every partial sum is an exact integer.
+@pytest.mark.parametrize("n", [1, 17, 100, 128, 129, 257, 300, 1000, 1100])
+def test_tc_backward_error_rodinia_matrix(rg, n):
+    A = synth.lud_rodinia_matrix(n)
+    assert _backward(A, _lu(rg, A, 128)) <= 1e-5, n
+
+
+@pytest.mark.parametrize("n", [300, 1024, 2048])
+def test_tc_forward_error_diag_dominant(rg, n):
+    A = synth.lud_diag_dominant(n)
+    L64, U64 = oracle.lud_unpack(oracle.lud(A))
+    p = _lu(rg, A, 128).cpu().numpy().astype(np.float64)
+    L, U = oracle.lud_unpack(p)
+    assert np.abs(L - L64).max() / np.abs(L64).max() <= 1e-5
+    assert np.abs(U - U64).max() / np.abs(U64).max() <= 1e-5
+
+
+@pytest.mark.parametrize("n", [7, 300, 512, 777])
+def test_tc_integer_factors_bit_exact(rg, n):
+    A, L0, U0 = synth.lud_integer_factors(n)
+    L, U = oracle.lud_unpack(_lu(rg, A, 128).cpu().numpy())
+    assert np.array_equal(L, L0) and np.array_equal(U, U0), n
+
+
+def test_tc_full_size_backward_error(rg):
+    # BASELINE configs[4] size (8192), Rodinia matrix; backward error via an fp64 product on
+    # the GPU (1.1e12 flop) on a row sample of A - L U
+    n = 8192
+    A = synth.lud_rodinia_matrix(n)
+    p = _lu(rg, A, 128).double()
+    L, U = _unpack_t(p)
+    rows = torch.arange(0, n, 61, device=p.device)
+    Ad = torch.from_numpy(A[rows.cpu().numpy()].astype(np.float64)).to(p.device)
+    err = float((Ad - L[rows] @ U).abs().max() / abs(A).max())
+    assert err <= 1e-5, err
