@@ -144,6 +144,9 @@ __device__ __forceinline__ void hs_ld(const float* __restrict__ base, int row, i
 // keeps each power row for the H steps during which levels 1..H read it (depth HsRing<H>::DP).
 // Rows outside [0, R) are zero-filled (their values only feed cells that are never stored).
 constexpr int HS_DT = 8;
+#ifndef RG_HS_TRAP
+#define RG_HS_TRAP 1  // top-halo trapezoid (hs_stream_step PRO); 0 only for A/B builds
+#endif
 template <int H>
 struct HsRing {
     static constexpr int need = HS_DT + H;
@@ -217,7 +220,13 @@ __device__ __forceinline__ void hs_issue_step(float* tring, float* pring, const 
     asm volatile("cp.async.commit_group;\n" ::);
 }
 
-template <int V, int H, int K, bool EC, bool ER>
+// PRO (the first 2H steps of a chunk): level l+1 is skipped at steps s < 2l+2.  Level L's rows
+// above y0-H+L are never needed (the output rows [y0, y1) depend on level L only through rows
+// [y0-H+L, y1+H-L)), and a skipped row is only ever read by rows that are skipped too, so the
+// stored results are unchanged; this trims the chunk's top halo from a rectangle of 2H rows per
+// level to the trapezoid (H(H+1) fewer row updates per chunk).  The bottom halo is already
+// trapezoidal through the one-row lag per level.
+template <int V, int H, int K, bool EC, bool ER, bool PRO>
 __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tring, float* pring,
                                                const float* __restrict__ tin, const float* __restrict__ pw,
                                                float* __restrict__ tout, int s, int ystart, int R, int C, int ylo,
@@ -233,6 +242,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
 
 #pragma unroll
     for (int l = 0; l < H; ++l) {
+        if (PRO && s < 2 * l + 2) break;  // levels l+1.. are all above their trapezoid (warp-uniform)
         const int g = g0 - l - 1;  // row computed by level l+1 (its power row was level 1's at step s-l)
         float pv[V];
         hs_read_row<V>(pring, sc0, (s - l) & (DP - 1), pv);
@@ -330,13 +340,19 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
     for (int k = 0; k < HS_DT - 1; ++k)
         hs_issue_step<V, H, EC, ER>(tring, pring, tin, pw, k, ystart, R, C, col0, sc0, tsrc, psrc);
     int s = 0;
-    for (; s + 3 <= nsteps; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 2, EC, ER>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    // prologue: the top-halo trapezoid (levels switched on two steps apart)
+    for (; RG_HS_TRAP && s + 3 <= nsteps && s < 2 * H; s += 3) {
+        hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 2, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
     }
-    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    for (; s + 3 <= nsteps; s += 3) {
+        hs_stream_step<V, H, 0, EC, ER, false>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 1, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 2, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    }
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
     asm volatile("cp.async.wait_group 0;\n" ::);  // drain before the rings are reused
 }
 
