@@ -410,6 +410,19 @@ def run_ours(args):
     else:
         g, tune_rows = rg.rodinia_tune("hotspot", N if ws == 1 else N // ws, N, iters, nranks=1, reps=2)
     t_tune = time.perf_counter() - t_tune
+    tuning = None
+    if tune_rows:
+        # heuristic pre-pruning: time only the 8 candidates the kernel-statistics
+        # model ranks best; regret = full-TDO median of its winner / full-TDO best
+        full = {tuple(r["g"]): r["median_ms"] for r in tune_rows if r["status"] == 0 and r["median_ms"] > 0}
+        t_pr = time.perf_counter()
+        gp, rows_p = rg.rodinia_tune_pruned("hotspot", N if ws == 1 else N // ws, N, iters, keep=8, reps=2)
+        t_pr = time.perf_counter() - t_pr
+        got = full.get(gp.astuple())
+        tuning = {"full": {"timed": len(full), "seconds": round(t_tune, 2), "best": list(g.astuple())},
+                  "pruned": {"keep": 8, "timed": sum(1 for r in rows_p if r["status"] == 0 and r["median_ms"] > 0),
+                             "seconds": round(t_pr, 2), "best": list(gp.astuple()),
+                             "regret": (got / min(full.values())) if got and full else None}}
 
     T, P = synth.hotspot_inputs(N, N)
     if ws == 1:
@@ -574,6 +587,7 @@ def run_ours(args):
             "speedup_vs_uncoarsened": speedups,
             "geomean_speedup_vs_uncoarsened": geomean,
             "workloads": extra,
+            "tuning": tuning,
             "paper_context": "27% Rodinia geomean speedup, A100/A4000, composite timing (PAPER.md:29)",
         }
         print(json.dumps(result), flush=True)

@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define RODINIA_ABI_VERSION 2
+#define RODINIA_ABI_VERSION 3
 
 typedef enum {
     RODINIA_OK = 0,
@@ -56,7 +56,9 @@ typedef enum {
     RODINIA_E_NODEV = -7,          /* no CUDA device / driver                                  */
     RODINIA_E_CUDA = -8,           /* CUDA runtime error (message in rodinia_last_error)       */
     RODINIA_E_NCCL = -9,           /* NCCL error or NCCL library not loadable                  */
-    RODINIA_E_NOMEM = -10          /* device or host allocation failed                         */
+    RODINIA_E_NOMEM = -10,         /* device or host allocation failed                         */
+    RODINIA_E_PRUNED = -11         /* tune row only: ranked below the `keep` best by the kernel-
+                                      statistics model of rodinia_tune_pruned, so never timed   */
 } rodinia_status;
 
 /* Granularity of one kernel launch (§V).
@@ -225,6 +227,8 @@ typedef struct {
     int32_t threads;         /* threads per CTA */
     int32_t ctas_per_sm;     /* occupancy (runtime query; 0 when no device) */
     int32_t status;          /* RODINIA_OK, or why the variant is pruned */
+    float model_ms;          /* kernel-statistics model estimate (rodinia_model_ms); -1 when the
+                                workload is not modelled or the row was not ranked */
 } rodinia_tune_row;
 
 /* Enumerate the instantiated variants of kernel k with their ptxas statistics and the
@@ -239,6 +243,28 @@ rodinia_status rodinia_variants(rodinia_kernel k, rodinia_tune_row* out, int32_t
 rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* p, int32_t reps,
                             rodinia_granularity* best, rodinia_tune_row* rows,
                             int32_t* nrows);
+
+/* Heuristic pre-pruning ("kernel statistics", the factor
+ * heuristics the paper leaves to future work).  Same as rodinia_tune, but every
+ * candidate that survives the compile-time filter is first ranked by rodinia_model_ms and only
+ * the `keep` best-ranked are timed; the others come back with status RODINIA_E_PRUNED and their
+ * model_ms.  Candidates the model cannot estimate (model_ms < 0: lud, pathfinder) are always
+ * timed.  keep <= 0 times every candidate (= rodinia_tune).  For hotspot the candidate set is
+ * the tuner's stage-2 block-factor sweep over every instantiation, not only the stage-1 top 4. */
+rodinia_status rodinia_tune_pruned(rodinia_kernel k, const rodinia_problem* p, int32_t reps,
+                                   int32_t keep, rodinia_granularity* best, rodinia_tune_row* rows,
+                                   int32_t* nrows);
+
+/* The model behind rodinia_tune_pruned, host-only (no device needed): estimates the time of one
+ * call of kernel k on problem p at row->g from closed-form work counts of the granularity
+ * (algorithmic HBM bytes incl. halo redundancy, issued lane-instructions incl. redundant halo
+ * updates, launches) and the ptxas statistics of the instantiation (registers, shared memory ->
+ * CTAs per SM -> latency-hiding factor), as a roofline max(bytes/BW, instructions/issue rate)
+ * divided by the occupancy factor plus a per-launch cost (DESIGN.md §5 "Pre-pruning").
+ * row->g, threads, regs, smem_bytes are inputs (ctas_per_sm too when > 0, else it is derived
+ * from regs/smem/threads); writes row->model_ms (-1 when the workload is not modelled).
+ * Device constants come from the current device when one exists, else B200 nominal values. */
+rodinia_status rodinia_model_ms(rodinia_kernel k, const rodinia_problem* p, rodinia_tune_row* row);
 
 /* Resolve what a NULL/zero granularity would run for this problem (cache or default). */
 rodinia_status rodinia_resolve(rodinia_kernel k, const rodinia_problem* p,

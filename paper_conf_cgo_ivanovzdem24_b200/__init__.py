@@ -36,6 +36,7 @@ RODINIA_E_NODEV = -7
 RODINIA_E_CUDA = -8
 RODINIA_E_NCCL = -9
 RODINIA_E_NOMEM = -10
+RODINIA_E_PRUNED = -11
 
 RODINIA_FAITHFUL = 1
 RODINIA_STREAM = 2
@@ -93,12 +94,13 @@ class TuneRow(ctypes.Structure):
     _fields_ = [("g", Granularity), ("median_ms", ctypes.c_float), ("regs", ctypes.c_int32),
                 ("spill_bytes", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
-                ("status", ctypes.c_int32)]
+                ("status", ctypes.c_int32), ("model_ms", ctypes.c_float)]
 
     def asdict(self):
         return dict(g=self.g.astuple(), median_ms=self.median_ms, regs=self.regs,
                     spill_bytes=self.spill_bytes, smem_bytes=self.smem_bytes,
-                    threads=self.threads, ctas_per_sm=self.ctas_per_sm, status=self.status)
+                    threads=self.threads, ctas_per_sm=self.ctas_per_sm, status=self.status,
+                    model_ms=self.model_ms)
 
 
 # ----------------------------------------------------------------------------- signatures
@@ -131,6 +133,9 @@ _SIGS = {
     "rodinia_variants": ([_i32, ctypes.POINTER(TuneRow), ctypes.POINTER(_i32)], _i32),
     "rodinia_tune": ([_i32, ctypes.POINTER(Problem), _i32, _PG, ctypes.POINTER(TuneRow),
                       ctypes.POINTER(_i32)], _i32),
+    "rodinia_tune_pruned": ([_i32, ctypes.POINTER(Problem), _i32, _i32, _PG, ctypes.POINTER(TuneRow),
+                             ctypes.POINTER(_i32)], _i32),
+    "rodinia_model_ms": ([_i32, ctypes.POINTER(Problem), ctypes.POINTER(TuneRow)], _i32),
     "rodinia_resolve": ([_i32, ctypes.POINTER(Problem), _PG], _i32),
     "rodinia_split_total": ([_i32, _i32, ctypes.POINTER(_i32)], _i32),
     "rodinia_slab": ([_i64, _i32, _i32, ctypes.POINTER(_i64), ctypes.POINTER(_i64)], _i32),
@@ -385,6 +390,30 @@ def rodinia_tune(kernel, rows: int, cols: int, iterations: int = 1, nranks: int 
     check(lib.rodinia_tune(_kernel(kernel), ctypes.byref(p), reps, ctypes.byref(best), out,
                            ctypes.byref(cap)), "rodinia_tune")
     return best, [out[i].asdict() for i in range(min(cap.value, 4096))]
+
+
+def rodinia_tune_pruned(kernel, rows: int, cols: int, iterations: int = 1, keep: int = 8, nranks: int = 1,
+                        reps: int = 3, depth: int = 0):
+    """Timing-driven selection after heuristic pre-pruning:
+    only the `keep` candidates the kernel-statistics model ranks best are timed."""
+    p = Problem(rows, cols, iterations, nranks, depth, 0)
+    best = Granularity()
+    cap = _i32(4096)
+    out = (TuneRow * cap.value)()
+    check(lib.rodinia_tune_pruned(_kernel(kernel), ctypes.byref(p), reps, keep, ctypes.byref(best), out,
+                                  ctypes.byref(cap)), "rodinia_tune_pruned")
+    return best, [out[i].asdict() for i in range(min(cap.value, 4096))]
+
+
+def rodinia_model_ms(kernel, g, rows: int, cols: int, iterations: int = 1, depth: int = 0, regs: int = -1,
+                     threads: int = 0, smem_bytes: int = 0, ctas_per_sm: int = 0, spill_bytes: int = 0) -> float:
+    """The pre-pruning model's estimate (ms) of one call at granularity g; -1 if not modelled."""
+    p = Problem(rows, cols, iterations, 1, depth, 0)
+    r = TuneRow()
+    r.g = g if isinstance(g, Granularity) else gran(*g) if isinstance(g, (tuple, list)) else gran(**g)
+    r.regs, r.threads, r.smem_bytes, r.ctas_per_sm, r.spill_bytes = regs, threads, smem_bytes, ctas_per_sm, spill_bytes
+    check(lib.rodinia_model_ms(_kernel(kernel), ctypes.byref(p), ctypes.byref(r)), "rodinia_model_ms")
+    return float(r.model_ms)
 
 
 def rodinia_resolve(kernel, rows: int, cols: int, iterations: int = 1, nranks: int = 1, depth: int = 0):

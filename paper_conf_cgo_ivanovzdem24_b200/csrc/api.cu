@@ -226,6 +226,7 @@ extern "C" const char* rodinia_status_string(rodinia_status s) {
         case RODINIA_E_CUDA: return "RODINIA_E_CUDA";
         case RODINIA_E_NCCL: return "RODINIA_E_NCCL";
         case RODINIA_E_NOMEM: return "RODINIA_E_NOMEM";
+        case RODINIA_E_PRUNED: return "RODINIA_E_PRUNED";
     }
     return "RODINIA_E_UNKNOWN";
 }

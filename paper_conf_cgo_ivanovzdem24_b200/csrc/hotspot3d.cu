@@ -431,6 +431,7 @@ rodinia_status tune_hotspot3d(const rodinia_problem& pr, int reps, rodinia_granu
             row.g.block_x = b.first;
             row.g.block_y = b.second;
             row.median_ms = -1.f;
+            row.model_ms = -1.f;
             const hotspot3d::Variant* v = nullptr;
             rodinia_status cs = hotspot3d::check(row.g, ny, &v);
             const PtxasStats* ps = find_stats(key);
@@ -441,6 +442,7 @@ rodinia_status tune_hotspot3d(const rodinia_problem& pr, int reps, rodinia_granu
                 row.ctas_per_sm = ctas_per_sm(fn, threads, 0);
                 cs = filter_decision(ps, threads, 0, 0);
             }
+            if (cs == RODINIA_OK) cs = prune_gate(RODINIA_HOTSPOT3D, pr, &row);
             if (cs == RODINIA_OK) {
                 std::vector<float> ts;
                 for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {

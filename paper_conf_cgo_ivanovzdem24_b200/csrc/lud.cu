@@ -628,6 +628,7 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
                 row.g.block_x = bx;
                 row.g.block_y = by;
                 row.median_ms = -1.f;
+                row.model_ms = -1.f;
                 lud::Plan pl;
                 rodinia_status cs = lud::plan(row.g, panel, &pl);
                 const PtxasStats* ps = find_stats(key);
@@ -642,6 +643,7 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
                     cs = filter_decision(ps, threads, (int)pl.smem, 0);
                     if (cs == RODINIA_OK && row.ctas_per_sm == 0) cs = RODINIA_E_FILTERED;
                 }
+                if (cs == RODINIA_OK) cs = prune_gate(RODINIA_LUD, pr, &row);
                 if (cs == RODINIA_OK) {
                     std::vector<float> ts;
                     for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {

@@ -439,6 +439,7 @@ rodinia_status tune_pathfinder(const rodinia_problem& pr, int reps, rodinia_gran
             memset(&row, 0, sizeof row);
             row.g = gran(g0.thread_x, 1, 1, 1, h, g0.index_mode, g0.flags);
             row.median_ms = -1.f;
+            row.model_ms = -1.f;
             pathfinder::Plan p;
             rodinia_status cs = pathfinder::plan(row.g, R, C, &p);
             const PtxasStats* ps = find_stats(key);
@@ -454,6 +455,7 @@ rodinia_status tune_pathfinder(const rodinia_problem& pr, int reps, rodinia_gran
                 row.ctas_per_sm = ctas_per_sm(fn, p.threads, row.smem_bytes);
                 cs = filter_decision(ps, p.threads, row.smem_bytes, 0);
             }
+            if (cs == RODINIA_OK) cs = prune_gate(RODINIA_PATHFINDER, pr, &row);
             if (cs == RODINIA_OK) {
                 std::vector<float> ts;
                 for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {

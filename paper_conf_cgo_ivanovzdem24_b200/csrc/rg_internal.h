@@ -84,6 +84,14 @@ rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p);
 // Cached device buffers of the *_host entry points (index 0..2), grown on demand.
 rodinia_status host_buffer(int i, size_t bytes, void** out);
 
+// ------------------------------------------------------------------ pre-pruning (tune.cu, model.cu)
+// Model estimate of one call at row.g (rodinia_model_ms); -1 when the workload is not modelled.
+float model_estimate_ms(rodinia_kernel k, const rodinia_problem& p, const rodinia_tune_row& row);
+// Called by every tuner after the compile-time filter, before timing a candidate: fills
+// row->model_ms and returns RODINIA_OK to time it or RODINIA_E_PRUNED (rodinia_tune_pruned).
+rodinia_status prune_gate(rodinia_kernel k, const rodinia_problem& p, rodinia_tune_row* row);
+bool prune_active();
+
 // ------------------------------------------------------------------ tune cache
 bool tune_cache_lookup(rodinia_kernel k, const rodinia_problem& p, rodinia_granularity* out);
 void tune_cache_store(rodinia_kernel k, const rodinia_problem& p, const rodinia_granularity& g,

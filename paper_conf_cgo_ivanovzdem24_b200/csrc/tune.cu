@@ -17,6 +17,8 @@ namespace rg {
 extern const PtxasStats kPtxasStats[];
 extern const int kNumPtxasStats;
 
+float model_estimate_ms(rodinia_kernel k, const rodinia_problem& p, const rodinia_tune_row& row);  // model.cu
+
 const PtxasStats* find_stats(const char* key) {
     for (int i = 0; i < kNumPtxasStats; ++i)
         if (strcmp(kPtxasStats[i].key, key) == 0) return &kPtxasStats[i];
@@ -66,6 +68,7 @@ static void fill_row(rodinia_kernel k, int i, bool have_dev, int base_spill, rod
     reg.info(i, &r->g, &fn, &key, &threads);
     const PtxasStats* st = find_stats(key);
     r->median_ms = -1.0f;
+    r->model_ms = -1.0f;
     r->regs = st ? st->regs : -1;
     r->spill_bytes = st ? st->spill_stores + st->spill_loads : -1;
     r->smem_bytes = st ? st->smem : -1;
@@ -103,6 +106,36 @@ rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
             return p.iterations == 32 ? gran(2, 4, 4, 2, 1, 1) : gran(4, 2, 2, 2, 1, 1);
     }
     return gran(1, 1, 1, 1, 1, 0);
+}
+
+// ---------------------------------------------------------------- pre-pruning gate
+// rodinia_tune_pruned runs a workload's tuner twice: a collect pass in which every candidate
+// that survives the compile-time filter is recorded with its model estimate and not timed, and
+// a select pass in which only the `keep` best-estimated candidates (and every candidate the
+// model cannot estimate) are timed.  Tuners call prune_gate() between the filter and timing.
+namespace {
+struct PruneState {
+    bool active = false, collect = false;
+    std::vector<rodinia_tune_row> seen;
+    std::vector<rodinia_granularity> keep;
+};
+thread_local PruneState g_prune;
+bool same_gran(const rodinia_granularity& a, const rodinia_granularity& b) { return memcmp(&a, &b, sizeof a) == 0; }
+}  // namespace
+
+bool prune_active() { return g_prune.active; }
+
+rodinia_status prune_gate(rodinia_kernel k, const rodinia_problem& p, rodinia_tune_row* row) {
+    row->model_ms = model_estimate_ms(k, p, *row);
+    if (!g_prune.active) return RODINIA_OK;
+    if (g_prune.collect) {
+        g_prune.seen.push_back(*row);
+        return RODINIA_E_PRUNED;
+    }
+    if (row->model_ms < 0) return RODINIA_OK;
+    for (const auto& g : g_prune.keep)
+        if (same_gran(g, row->g)) return RODINIA_OK;
+    return RODINIA_E_PRUNED;
 }
 
 // ---------------------------------------------------------------- synthetic data
@@ -194,6 +227,7 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
         memset(&row, 0, sizeof row);
         row.g = gc;
         row.median_ms = -1.f;
+        row.model_ms = -1.f;
         const hotspot::DirectVariant* dv;
         const hotspot::StreamVariant* sv;
         rodinia_status cs = hotspot::check(row.g, R, C, &dv, &sv);
@@ -218,6 +252,7 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
                 }
             }
         }
+        if (cs == RODINIA_OK) cs = prune_gate(RODINIA_HOTSPOT, p, &row);
         if (cs == RODINIA_OK) {
             std::vector<float> ts;
             for (int r = -1; r < reps && cs == RODINIA_OK; ++r) {
@@ -248,6 +283,15 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
     for (auto& r : *rows) if (r.status == RODINIA_OK && r.median_ms > 0) ok.push_back(r);
     std::sort(ok.begin(), ok.end(), [](const rodinia_tune_row& a, const rodinia_tune_row& b) { return a.median_ms < b.median_ms; });
     std::vector<rodinia_granularity> tops;
+    if (prune_active()) {
+        // pre-pruning: the model ranks the block-factor sweep of every instantiation
+        for (auto& g : stage1) {
+            bool dup = false;
+            for (auto& t : tops) dup = dup || same_instantiation(t, g);
+            if (!dup) tops.push_back(g);
+        }
+        ok.clear();
+    }
     for (auto& r : ok) {
         bool dup = false;
         for (auto& t : tops) dup = dup || same_instantiation(t, r.g);
@@ -313,6 +357,61 @@ extern "C" rodinia_status rodinia_tune(rodinia_kernel k, const rodinia_problem* 
         case RODINIA_HOTSPOT3D: st = tune_hotspot3d(*p, reps, best, &out); break;
         default: st = tune_lud(*p, reps, best, &out); break;
     }
+    if (nrows) {
+        const int cap = *nrows;
+        for (int i = 0; i < cap && i < (int)out.size(); ++i) rows[i] = out[i];
+        *nrows = (int)out.size();
+    }
+    return st;
+}
+
+static rodinia_status run_tuner(rodinia_kernel k, const rodinia_problem& p, int reps, rodinia_granularity* best,
+                                std::vector<rodinia_tune_row>* out) {
+    switch (k) {
+        case RODINIA_HOTSPOT: return tune_hotspot(p, reps, best, out);
+        case RODINIA_SRAD: return tune_srad(p, reps, best, out);
+        case RODINIA_PATHFINDER: return tune_pathfinder(p, reps, best, out);
+        case RODINIA_HOTSPOT3D: return tune_hotspot3d(p, reps, best, out);
+        default: return tune_lud(p, reps, best, out);
+    }
+}
+
+extern "C" rodinia_status rodinia_tune_pruned(rodinia_kernel k, const rodinia_problem* p, int32_t reps, int32_t keep,
+                                              rodinia_granularity* best, rodinia_tune_row* rows, int32_t* nrows) {
+    if (keep <= 0) return rodinia_tune(k, p, reps, best, rows, nrows);
+    if (!p || !best || reps < 1 || p->rows < 1 || p->cols < 1 || p->iterations < 0 || p->nranks < 1)
+        return set_error(RODINIA_E_INVALID, "tune_pruned: bad arguments");
+    if (nrows && *nrows > 0 && !rows) return set_error(RODINIA_E_INVALID, "tune_pruned: rows is null");
+    if ((int)k < 0 || (int)k > 4) return set_error(RODINIA_E_INVALID, "tune_pruned: unknown kernel %d", (int)k);
+    DeviceInfo di;
+    RG_TRY(device_info(&di));
+    // collect pass: every filter survivor with its model estimate, nothing timed
+    g_prune = PruneState();
+    g_prune.active = true;
+    g_prune.collect = true;
+    std::vector<rodinia_tune_row> scratch;
+    rodinia_granularity dummy;
+    rodinia_status st = run_tuner(k, *p, reps, &dummy, &scratch);
+    if (st != RODINIA_OK && st != RODINIA_E_FILTERED) {
+        g_prune = PruneState();
+        return st;
+    }
+    clear_error();
+    std::vector<rodinia_tune_row> ranked;
+    for (auto& r : g_prune.seen)
+        if (r.model_ms >= 0) ranked.push_back(r);
+    std::stable_sort(ranked.begin(), ranked.end(),
+                     [](const rodinia_tune_row& a, const rodinia_tune_row& b) { return a.model_ms < b.model_ms; });
+    for (size_t i = 0; i < ranked.size() && (int)g_prune.keep.size() < keep; ++i) {
+        bool dup = false;
+        for (auto& g : g_prune.keep) dup = dup || same_gran(g, ranked[i].g);
+        if (!dup) g_prune.keep.push_back(ranked[i].g);
+    }
+    // select pass: time the kept candidates (and every unmodelled one)
+    g_prune.collect = false;
+    std::vector<rodinia_tune_row> out;
+    st = run_tuner(k, *p, reps, best, &out);
+    g_prune = PruneState();
     if (nrows) {
         const int cap = *nrows;
         for (int i = 0; i < cap && i < (int)out.size(); ++i) rows[i] = out[i];

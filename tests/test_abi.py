@@ -29,7 +29,7 @@ def test_every_header_symbol_exported():
     for n in names:
         assert hasattr(rg.lib, n), n
     assert set(names) == set(rg.EXPORTED)
-    assert rg.lib.rodinia_abi_version() == 2
+    assert rg.lib.rodinia_abi_version() == 3
 
 
 def test_status_strings():

@@ -83,3 +83,36 @@ def test_variant_tables_agree_with_runtime(rg):
         for r in rows:
             if r["status"] == 0:
                 assert r["ctas_per_sm"] >= 1 and r["spill_bytes"] == 0, (k, r)
+
+
+def _timed(rows):
+    return {tuple(r["g"]): r["median_ms"] for r in rows if r["status"] == 0 and r["median_ms"] > 0}
+
+
+@pytest.mark.parametrize("kernel,shape", [("hotspot", dict(rows=8192, cols=8192, iterations=48)),
+                                          ("srad", dict(rows=8192, cols=8192, iterations=10)),
+                                          ("hotspot3d", dict(rows=1024, cols=1024, iterations=4, depth=64))])
+def test_pruned_tune_times_only_keep_and_finds_a_near_best(rg, kernel, shape):
+    """Heuristic pre-pruning: only `keep` candidates are timed; the rest carry
+    RODINIA_E_PRUNED and a model estimate; the winner is within 25 % of full TDO's winner (the
+    tune table's own run-to-run noise under the power cap is ~10 %)."""
+    keep = 8
+    best_full, rows_full = rg.rodinia_tune(kernel, reps=3, **shape)
+    best_p, rows_p = rg.rodinia_tune_pruned(kernel, keep=keep, reps=3, **shape)
+    timed_p = _timed(rows_p)
+    assert 1 <= len(timed_p) <= keep
+    assert len(_timed(rows_full)) > keep
+    assert any(r["status"] == rg.RODINIA_E_PRUNED for r in rows_p)
+    assert all(r["model_ms"] > 0 for r in rows_p if r["status"] in (0, rg.RODINIA_E_PRUNED))
+    full = _timed(rows_full)
+    ref = min(full.values())
+    got = full.get(best_p.astuple(), timed_p[best_p.astuple()])
+    assert got <= 1.25 * ref, (best_p.astuple(), got, best_full.astuple(), ref)
+
+
+def test_pruned_tune_keeps_unmodelled_workloads_exhaustive(rg):
+    # pathfinder is not modelled (latency chain): every filter survivor is still timed
+    _, rows_full = rg.rodinia_tune("pathfinder", 100, 20000, reps=1)
+    _, rows_p = rg.rodinia_tune_pruned("pathfinder", 100, 20000, keep=2, reps=1)
+    assert len(_timed(rows_p)) == len(_timed(rows_full))
+    assert all(r["model_ms"] == -1 for r in rows_p)
