@@ -197,7 +197,9 @@ rodinia_status rodinia_pathfinder_host(const int32_t* wall, int64_t rows, int64_
 /* ---------------------------------------------------------------------------------------
  * lud -- Rodinia lud (blocked Doolittle LU, no pivoting), L1-L6.  a (n x n fp32)
  * is factored in place: unit-diagonal L strictly below the diagonal, U on and above.
- * panel: block (panel) width; 16 = Rodinia's BLOCK_SIZE (0 => 16).  Supported: 16, 32.
+ * panel: block (panel) width; 16 = Rodinia's BLOCK_SIZE (0 => 16).  Supported: 16, 32, and
+ * 128 = two-level blocking (inner panel 32) whose rank-128 trailing updates run on the tensor
+ * cores (tcgen05.mma kind::tf32 with the 3xTF32 split; g is ignored there).
  * The panel width changes fp32 rounding order and is reported separately from coarsening
  * (reading L5).  Zero pivots give inf/NaN (no pivoting, as Rodinia). */
 rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
