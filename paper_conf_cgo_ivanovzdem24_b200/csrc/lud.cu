@@ -358,7 +358,7 @@ __global__ void __launch_bounds__(256)
 
 namespace tc {
 // Whole factorisation, 128-wide outer blocks (inner panel 32).  Returns the launch count.
-inline int launch_all(float* const* slot, int n, cudaStream_t s) {
+inline int launch_all(float* const* slot, int n, float* img_a, float* img_b, cudaStream_t s) {
     constexpr int NB = 128, P = 32;
     const int m32 = (n + P - 1) / P;
     int launches = 0;
@@ -374,14 +374,14 @@ inline int launch_all(float* const* slot, int n, cudaStream_t s) {
             if (a < e) {
                 // rank-32 update restricted to the outer block's L-shaped panel region
                 const Rect rs[2] = {make_rect(a, a, n - a, e - a, p0, P), make_rect(a, e, e - a, n - e, p0, P)};
-                launch_update(slot, n, rs, 2, s);
-                ++launches;
+                launch_update2(slot, n, rs, 2, a, img_a, img_b, s);
+                launches += 3;
             }
         }
         if (e < n) {  // rank-128 trailing update on the tensor cores
             const Rect r = make_rect(e, e, n - e, n - e, o, e - o);
-            launch_update(slot, n, &r, 1, s);
-            ++launches;
+            launch_update2(slot, n, &r, 1, e, img_a, img_b, s);
+            launches += 3;
         }
     }
     return launches;
@@ -446,7 +446,7 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
         pl->v = nullptr;
         pl->sv = nullptr;
         pl->bx = pl->by = 1;
-        pl->smem = tc::smem_bytes(tc::KC_MAIN);
+        pl->smem = tc::smem_bytes2();
         return RODINIA_OK;
     }
     if (g.index_mode != 0 && g.index_mode != 1)
@@ -504,6 +504,7 @@ static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
 struct GraphEntry {
     cudaGraphExec_t exec = nullptr;
     float** slot = nullptr;
+    float* img = nullptr;   // panel-128 path: the two tensor-core operand images
     int launches = 0;
 };
 static std::mutex g_mu;
@@ -520,8 +521,9 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
     const int m = (n + pl.p - 1) / pl.p;
     if (!ge.exec) {
         RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
-        const void* ifn = pl.tc ? (const void*)tc::lud_tc_update<tc::KC_MAIN>
+        const void* ifn = pl.tc ? (const void*)tc::lud_tc_update2
                                 : pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
+        if (pl.tc) RG_CUDA(cudaMalloc(&ge.img, 2 * tc::img_floats(n) * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
         cudaStream_t cs;
@@ -529,7 +531,7 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         cudaGraph_t graph;
         RG_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
         int nl = 3 * m - 2;
-        if (pl.tc) nl = tc::launch_all(ge.slot, n, cs);
+        if (pl.tc) nl = tc::launch_all(ge.slot, n, ge.img, ge.img + tc::img_floats(n), cs);
         else launch_all(pl, ge.slot, n, cs);
         cudaError_t e = cudaStreamEndCapture(cs, &graph);
         cudaStreamDestroy(cs);
