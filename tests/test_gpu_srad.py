@@ -75,14 +75,15 @@ def _stream_grans(rg):
     return out
 
 
-@pytest.mark.parametrize("R,C", [(131, 97), (70, 256), (33, 260)])
-def test_all_variants_bit_identical(rg, R, C):
+@pytest.mark.parametrize("R,C,niter", [(131, 97, 6), (70, 256, 6), (33, 260, 6), (300, 516, 7), (181, 260, 5)])
+def test_all_variants_bit_identical(rg, R, C, niter):
+    # 300 x 516 has interior chunks/bands (the stream family's fast path) next to edge ones
     J = synth.srad_input(R, C, seed=3)
     roi = (0, min(60, R - 1), 5, 70)
-    base = _run(rg, J, roi, 0.5, 6, UNC)
-    assert rel_err(base, oracle.srad(J, *roi, 0.5, 6)) <= TOL
+    base = _run(rg, J, roi, 0.5, niter, UNC)
+    assert rel_err(base, oracle.srad(J, *roi, 0.5, niter)) <= TOL
     for g in _fused_grans() + _stream_grans(rg):
-        assert np.array_equal(_run(rg, J, roi, 0.5, 6, g), base), g
+        assert np.array_equal(_run(rg, J, roi, 0.5, niter, g), base), g
 
 
 def test_uniform_and_lambda_zero_unchanged(rg):
@@ -93,11 +94,12 @@ def test_uniform_and_lambda_zero_unchanged(rg):
     assert np.array_equal(_run(rg, J, (0, 20, 0, 20), 0.0, 5, (2, 2, 1, 1, 1, 0, 0)), J)
 
 
-def test_degenerate_roi_reported(rg):
+@pytest.mark.parametrize("g", [UNC, (4, 1, 1, 1, 1, 1, 2)])
+def test_degenerate_roi_reported(rg, g):
     J = synth.srad_input(40, 40)
     J[:4, :4] = 0.0
     t = torch.from_numpy(J).cuda()
-    rg.rodinia_srad(t, 0, 3, 0, 3, 0.5, 3, g=UNC)  # asynchronous: returns before the check
+    rg.rodinia_srad(t, 0, 3, 0, 3, 0.5, 3, g=g)  # asynchronous: returns before the check
     with pytest.raises(rg.RodiniaError) as e:
         rg.rodinia_sync()
     assert e.value.status == rg.RODINIA_E_DEGENERATE
