@@ -133,6 +133,19 @@ rodinia_status rodinia_hotspot_host(const float* temp_in, const float* power, fl
                                     const rodinia_hotspot_coeffs* coeffs,
                                     const rodinia_granularity* g, void* stream);
 
+/* A batch of `count` independent problems with HOST buffers: problem i reads temp_in[i] and
+ * power[i] and writes temp_out[i] (each rows x cols; arrays of `count` host pointers).  Two
+ * library-owned device buffer sets are pipelined: the H2D copies of problem i+1 and the D2H
+ * copy of problem i-1 run on copy streams while problem i is solved on `stream` (events
+ * order reuse of a set).  Synchronous: returns when every result is in host memory.  The
+ * copies overlap compute only if the host buffers are pinned.  Per problem the arithmetic is
+ * exactly rodinia_hotspot's. */
+rodinia_status rodinia_hotspot_host_batch(const float* const* temp_in, const float* const* power,
+                                          float* const* temp_out, int32_t count, int64_t rows,
+                                          int64_t cols, int32_t iterations,
+                                          const rodinia_hotspot_coeffs* coeffs,
+                                          const rodinia_granularity* g, void* stream);
+
 /* ---------------------------------------------------------------------------------------
  * hotspot3d -- Rodinia hotspot3D `hotspotOpt1` (7-point 3-D thermal stencil, named in
  * PAPER.md:395), readings T1-T4.  Grid nx (x, fastest) x ny x nz,

@@ -119,6 +119,8 @@ _SIGS = {
     "rodinia_hotspot_coeffs_rodinia": ([_i64, _i64, _f64, _f64, _PC], _i32),
     "rodinia_hotspot": ([_vp, _vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
     "rodinia_hotspot_host": ([_vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
+    "rodinia_hotspot_host_batch": ([ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i64, _i64,
+                                    _i32, _PC, _PG, _vp], _i32),
     "rodinia_hotspot3d_coeffs_rodinia": ([_i64, _i64, _i64, _f64, _f64, _f64, ctypes.c_void_p], _i32),
     "rodinia_hotspot3d": ([_vp, _vp, _vp, _vp, _i64, _i64, _i64, _i32, _vp, _PG, _vp], _i32),
     "rodinia_hotspot3d_host": ([_vp, _vp, _vp, _i64, _i64, _i64, _i32, _vp, _PG, _vp], _i32),
@@ -231,6 +233,27 @@ def rodinia_hotspot(temp, power, iterations: int, coeffs=None, g=None, out=None,
         _stream(stream))
     check(st, "rodinia_hotspot")
     return out
+
+
+def rodinia_hotspot_host_batch(temps, powers, iterations: int, coeffs=None, g=None, outs=None, stream=None):
+    """Batch of independent problems with host buffers (numpy float32, ideally pinned): copies
+    of neighbouring problems overlap the solves (two device buffer sets).  Returns the outputs."""
+    import numpy as np
+    ts = [np.ascontiguousarray(t, dtype=np.float32) for t in temps]
+    ps = [np.ascontiguousarray(p, dtype=np.float32) for p in powers]
+    if len(ts) != len(ps) or not ts:
+        raise ValueError("temps and powers must be non-empty lists of equal length")
+    R, C = ts[0].shape
+    if any(t.shape != (R, C) for t in ts + ps):
+        raise ValueError("all problems must have the same shape")
+    if outs is None:
+        outs = [np.empty_like(ts[0]) for _ in ts]
+    n = len(ts)
+    arr = lambda xs: (_vp * n)(*[x.ctypes.data for x in xs])
+    st = lib.rodinia_hotspot_host_batch(arr(ts), arr(ps), arr(outs), n, R, C, int(iterations),
+                                        None if coeffs is None else ctypes.byref(coeffs), _g(g), _stream(stream))
+    check(st, "rodinia_hotspot_host_batch")
+    return outs
 
 
 def rodinia_hotspot_host(temp, power, iterations: int, coeffs=None, g=None, out=None,

@@ -388,9 +388,12 @@ extern "C" rodinia_status rodinia_hotspot(const float* tin, const float* p, floa
 namespace rg {
 struct HostStage {
     std::mutex mu;
-    void* buf[3] = {nullptr, nullptr, nullptr};
-    size_t cap[3] = {0, 0, 0};
-    int dev[3] = {-1, -1, -1};
+    void* buf[9] = {nullptr};   // 0..2: *_host calls; 3..8: two buffer sets of the batch call
+    size_t cap[9] = {0};
+    int dev[9] = {-1, -1, -1, -1, -1, -1, -1, -1, -1};
+    cudaStream_t h2d = nullptr, d2h = nullptr;  // copy streams of rodinia_hotspot_host_batch
+    cudaEvent_t ev[6] = {nullptr};              // per set: inputs landed, solved, result read
+    int sdev = -1;
 };
 HostStage& host_stage() {
     static HostStage hs;
@@ -431,6 +434,58 @@ extern "C" rodinia_status rodinia_hotspot_host(const float* tin, const float* p,
     RG_CUDA(cudaMemcpyAsync(dp, p, bytes, cudaMemcpyHostToDevice, s));
     RG_TRY(rodinia_hotspot((const float*)dt, (const float*)dp, (float*)dout, nullptr, R, C, iters, coeffs, g, stream));
     RG_CUDA(cudaMemcpyAsync(tout, dout, bytes, cudaMemcpyDeviceToHost, s));
+    RG_CUDA(cudaStreamSynchronize(s));
+    return RODINIA_OK;
+}
+
+extern "C" rodinia_status rodinia_hotspot_host_batch(const float* const* tin, const float* const* p,
+                                                     float* const* tout, int32_t count, int64_t R, int64_t C,
+                                                     int32_t iters, const rodinia_hotspot_coeffs* coeffs,
+                                                     const rodinia_granularity* g, void* stream) {
+    if (count < 0 || (count > 0 && (!tin || !p || !tout)))
+        return set_error(RODINIA_E_INVALID, "hotspot_host_batch: bad arguments");
+    for (int i = 0; i < count; ++i) RG_TRY(hotspot_validate(tin[i], p[i], tout[i], R, C, iters, coeffs));
+    if (count == 0) return RODINIA_OK;
+    DeviceInfo di;
+    RG_TRY(device_info(&di));
+    HostStage& hs = host_stage();
+    std::lock_guard<std::mutex> lk(hs.mu);
+    if (hs.sdev != di.device) {
+        RG_CUDA(cudaStreamCreateWithFlags(&hs.h2d, cudaStreamNonBlocking));
+        RG_CUDA(cudaStreamCreateWithFlags(&hs.d2h, cudaStreamNonBlocking));
+        for (auto& e : hs.ev) RG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        hs.sdev = di.device;
+    }
+    const size_t bytes = (size_t)R * C * sizeof(float);
+    void* dv[2][3];
+    for (int b = 0; b < 2; ++b)
+        for (int k = 0; k < 3; ++k) RG_TRY(host_buffer(3 + 3 * b + k, bytes, &dv[b][k]));
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaEvent_t* in_ready = hs.ev;        // [2]: H2D of the set's inputs done
+    cudaEvent_t* solved = hs.ev + 2;      // [2]: solve done (inputs free, output valid)
+    cudaEvent_t* read = hs.ev + 4;        // [2]: D2H of the set's output done
+    auto h2d = [&](int i) -> rodinia_status {
+        const int b = i & 1;
+        if (i >= 2) RG_CUDA(cudaStreamWaitEvent(hs.h2d, solved[b], 0));  // problem i-2 done with the set
+        RG_CUDA(cudaMemcpyAsync(dv[b][0], tin[i], bytes, cudaMemcpyHostToDevice, hs.h2d));
+        RG_CUDA(cudaMemcpyAsync(dv[b][1], p[i], bytes, cudaMemcpyHostToDevice, hs.h2d));
+        RG_CUDA(cudaEventRecord(in_ready[b], hs.h2d));
+        return RODINIA_OK;
+    };
+    RG_TRY(h2d(0));
+    for (int i = 0; i < count; ++i) {
+        const int b = i & 1;
+        if (i + 1 < count) RG_TRY(h2d(i + 1));  // next inputs stream in while problem i solves
+        RG_CUDA(cudaStreamWaitEvent(s, in_ready[b], 0));
+        if (i >= 2) RG_CUDA(cudaStreamWaitEvent(s, read[b], 0));  // output of problem i-2 read back
+        RG_TRY(rodinia_hotspot((const float*)dv[b][0], (const float*)dv[b][1], (float*)dv[b][2], nullptr, R, C, iters,
+                               coeffs, g, stream));
+        RG_CUDA(cudaEventRecord(solved[b], s));
+        RG_CUDA(cudaStreamWaitEvent(hs.d2h, solved[b], 0));  // result of problem i streams out
+        RG_CUDA(cudaMemcpyAsync(tout[i], dv[b][2], bytes, cudaMemcpyDeviceToHost, hs.d2h));
+        RG_CUDA(cudaEventRecord(read[b], hs.d2h));
+    }
+    RG_CUDA(cudaStreamSynchronize(hs.d2h));
     RG_CUDA(cudaStreamSynchronize(s));
     return RODINIA_OK;
 }

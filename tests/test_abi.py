@@ -121,3 +121,12 @@ def test_split_total_footnote_examples():
         assert x * y * z == t and max(x, y, z) <= t
     with pytest.raises(rg.RodiniaError):
         rg.rodinia_split_total(0, 3)
+
+
+def test_hotspot_host_batch_argument_validation_without_device():
+    null3 = (ctypes.c_void_p * 1)(None)
+    ok = (ctypes.c_void_p * 1)(1)
+    assert rg.lib.rodinia_hotspot_host_batch(ok, ok, ok, -1, 8, 8, 1, None, None, None) == rg.RODINIA_E_INVALID
+    assert rg.lib.rodinia_hotspot_host_batch(null3, ok, ok, 1, 8, 8, 1, None, None, None) == rg.RODINIA_E_INVALID
+    assert rg.lib.rodinia_hotspot_host_batch(ok, ok, ok, 1, 0, 8, 1, None, None, None) == rg.RODINIA_E_INVALID
+    assert rg.lib.rodinia_hotspot_host_batch(None, None, None, 0, 8, 8, 1, None, None, None) == rg.RODINIA_OK

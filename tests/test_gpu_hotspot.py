@@ -141,3 +141,14 @@ def test_variant_stats_match_runtime_attributes(rg):
     rows = rg.rodinia_variants("hotspot")
     assert rows and all(r["regs"] > 0 for r in rows)
     assert all(r["ctas_per_sm"] >= 1 for r in rows if r["status"] == 0)
+
+
+def test_host_batch_pipelined_equals_single_calls(rg):
+    # rodinia_hotspot_host_batch overlaps copies with solves (two device buffer sets): every
+    # problem's result is bitwise the single-call result; 3 problems exercise set reuse
+    c = rg.rodinia_hotspot_coeffs_rodinia(200, 300, 200 * 31.25e-6, 300 * 31.25e-6)
+    ins = [synth.hotspot_inputs(200, 300, seed_t=10 + i, seed_p=20 + i) for i in range(3)]
+    g = (4, 1, 1, 2, 8, 1, rg.RODINIA_STREAM)
+    outs = rg.rodinia_hotspot_host_batch([t for t, _ in ins], [p for _, p in ins], 19, coeffs=c, g=g)
+    for (t, p), o in zip(ins, outs):
+        assert np.array_equal(o, rg.rodinia_hotspot_host(t, p, 19, coeffs=c, g=g))
