@@ -41,7 +41,7 @@ namespace srad {
 typedef void (*FusedFn)(const float*, float*, int, int, int, int, float, const SradIter*);
 struct Variant { int tx, ty, mode; FusedFn fn; const char* key; };
 typedef void (*StreamFn)(const float*, float*, int, int, int, int, float, const SradIter*, int);
-struct StreamVariant { int v; StreamFn fn; const char* key; };
+struct StreamVariant { int v, occ; StreamFn fn; const char* key; };
 // Plan: dataflow (uncoarsened) iff granularity is exactly the uncoarsened one.
 struct Plan {
     bool dataflow;
