@@ -135,34 +135,54 @@ __global__ void __launch_bounds__(256)
             }
         }
     };
-    float B[TY][TX], Cc[TY][TX], T[TY][TX];
+    float B[TY][TX], Cc[TY][TX], T[TY][TX], P[TY][TX];
     load_cells(0, Cc, tin);
 #pragma unroll
     for (int j = 0; j < TY; ++j)
 #pragma unroll
         for (int i = 0; i < TX; ++i) B[j][i] = Cc[j][i];
     load_cells(min(1, nz - 1), T, tin);
-    // halo ring of the tile: left/right columns (SY cells each) and top/bottom rows (OX each)
-    const int nhalo = 2 * SY + 2 * OX;
+    load_cells(0, P, pw);
+    // halo ring of the tile: left/right columns (SY cells each) and top/bottom rows (OX each);
+    // thread t owns ring cells t, t+256, ... and keeps the next plane's values in registers
+    constexpr int NHALO = 2 * SY + 2 * OX, NH = (NHALO + 255) / 256;
+    int hoff[NH], hsy[NH], hsx[NH];
+#pragma unroll
+    for (int q = 0; q < NH; ++q) {
+        const int h = threadIdx.x + 256 * q;
+        int sy = 0, sx = 0;
+        if (h < SY) { sy = h; sx = 0; }
+        else if (h < 2 * SY) { sy = h - SY; sx = SX - 1; }
+        else if (h < 2 * SY + OX) { sy = 0; sx = 1 + (h - 2 * SY); }
+        else if (h < NHALO) { sy = SY - 1; sx = 1 + (h - 2 * SY - OX); }
+        hsy[q] = sy; hsx[q] = sx;
+        const int gy = min(max(y0 - 1 + sy, 0), ny - 1), gx = min(max(x0 - 1 + sx, 0), nx - 1);
+        hoff[q] = gy * nx + gx;
+    }
+    float hv[NH];
+#pragma unroll
+    for (int q = 0; q < NH; ++q) hv[q] = threadIdx.x + 256 * q < NHALO ? __ldg(tin + hoff[q]) : 0.f;
     for (int z = 0; z < nz; ++z) {
         const int buf = z & 1;
-        const float* pz = tin + (size_t)z * plane;
 #pragma unroll
         for (int j = 0; j < TY; ++j)
 #pragma unroll
             for (int i = 0; i < TX; ++i) pl[buf][1 + ty * TY + j][1 + tx * TX + i] = Cc[j][i];
-        for (int h = threadIdx.x; h < nhalo; h += 256) {
-            int sy, sx;
-            if (h < SY) { sy = h; sx = 0; }
-            else if (h < 2 * SY) { sy = h - SY; sx = SX - 1; }
-            else if (h < 2 * SY + OX) { sy = 0; sx = 1 + (h - 2 * SY); }
-            else { sy = SY - 1; sx = 1 + (h - 2 * SY - OX); }
-            const int gy = min(max(y0 - 1 + sy, 0), ny - 1), gx = min(max(x0 - 1 + sx, 0), nx - 1);
-            pl[buf][sy][sx] = __ldg(pz + (size_t)gy * nx + gx);
-        }
-        float P[TY][TX];
-        load_cells(z, P, pw);
+#pragma unroll
+        for (int q = 0; q < NH; ++q)
+            if (threadIdx.x + 256 * q < NHALO) pl[buf][hsy[q]][hsx[q]] = hv[q];
         __syncthreads();
+        // the next plane's global loads are issued before this plane's arithmetic (one plane of
+        // lookahead for T, P and the halo ring), so their latency hides behind the compute
+        float T2[TY][TX], P2[TY][TX], hv2[NH];
+        const bool more = z + 1 < nz;
+        if (more) {
+            load_cells(min(z + 2, nz - 1), T2, tin);
+            load_cells(z + 1, P2, pw);
+            const float* pz1 = tin + (size_t)(z + 1) * plane;
+#pragma unroll
+            for (int q = 0; q < NH; ++q) hv2[q] = threadIdx.x + 256 * q < NHALO ? __ldg(pz1 + hoff[q]) : 0.f;
+        }
 #pragma unroll
         for (int j = 0; j < TY; ++j) {
             const int ly = 1 + ty * TY + j;
@@ -192,12 +212,16 @@ __global__ void __launch_bounds__(256)
                 }
             }
         }
-        // advance the z window (T of plane z+2, clamped)
+        if (more) {  // advance the z window
 #pragma unroll
-        for (int j = 0; j < TY; ++j)
+            for (int j = 0; j < TY; ++j)
 #pragma unroll
-            for (int i = 0; i < TX; ++i) { B[j][i] = Cc[j][i]; Cc[j][i] = T[j][i]; }
-        if (z + 1 < nz) load_cells(min(z + 2, nz - 1), T, tin);
+                for (int i = 0; i < TX; ++i) {
+                    B[j][i] = Cc[j][i]; Cc[j][i] = T[j][i]; T[j][i] = T2[j][i]; P[j][i] = P2[j][i];
+                }
+#pragma unroll
+            for (int q = 0; q < NH; ++q) hv[q] = hv2[q];
+        }
     }
 }
 
