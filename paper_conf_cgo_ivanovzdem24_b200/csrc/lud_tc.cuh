@@ -469,6 +469,8 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
 
 constexpr size_t smem_bytes2() { return (size_t)NS2 * 4 * BM * KC2 * 4 + 128; }
 
+// v1 (single-thread-group staging, kept as the reference the layout probe
+// tools/ubench/tc_dump.cu exercises; the library runs lud_tc_update2 above).
 #ifndef RG_LUD_KC
 #define RG_LUD_KC 16
 #endif
