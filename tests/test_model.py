@@ -123,3 +123,18 @@ def test_unmodelled_workloads_and_errors():
         _m("hotspot", (0, 1, 1, 1, 1, 0, 0), rows=N, cols=N)
     with pytest.raises(rg.RodiniaError):
         _m("hotspot", (1, 1, 1, 1, 1, 0, 0), rows=0, cols=N)
+
+
+def test_tune_pruned_argument_validation():
+    import ctypes
+    import torch
+    p = rg.Problem(256, 256, 16, 1, 0, 0)
+    best = rg.Granularity()
+    n = ctypes.c_int32(0)
+    # bad arguments are rejected before any device work
+    assert rg.lib.rodinia_tune_pruned(0, None, 1, 4, ctypes.byref(best), None, ctypes.byref(n)) == rg.RODINIA_E_INVALID
+    assert rg.lib.rodinia_tune_pruned(0, ctypes.byref(p), 0, 4, ctypes.byref(best), None, ctypes.byref(n)) == rg.RODINIA_E_INVALID
+    assert rg.lib.rodinia_tune_pruned(9, ctypes.byref(p), 1, 4, ctypes.byref(best), None, ctypes.byref(n)) == rg.RODINIA_E_INVALID
+    if not torch.cuda.is_available():
+        st = rg.lib.rodinia_tune_pruned(0, ctypes.byref(p), 1, 4, ctypes.byref(best), None, ctypes.byref(n))
+        assert st == rg.RODINIA_E_NODEV
