@@ -141,8 +141,11 @@ __global__ void __launch_bounds__(256)
 // rows stream through a per-lane cp.async ring in shared memory PfRing::D-1 rows ahead.  The band's
 // halo is h rounded up to 4 columns per side (keeps 16-byte alignment).
 // ring depth (rows in flight); deeper rings (16-32) were measured slower (longer prologue)
+#ifndef RG_PF_D
+#define RG_PF_D 8  // A/B builds only (tools/build_lib.py --define RG_PF_D=16)
+#endif
 template <int CELLS>
-struct PfRing { static constexpr int D = 8; };
+struct PfRing { static constexpr int D = RG_PF_D * CELLS <= 256 ? RG_PF_D : 256 / CELLS; };  // <= 32 KiB static smem
 
 template <int CELLS, bool EC>
 __device__ __forceinline__ void pf_issue(int32_t* ring, const int32_t* __restrict__ wall, int row, int C,
