@@ -147,14 +147,25 @@ __global__ void __launch_bounds__(256)
 template <int CELLS>
 struct PfRing { static constexpr int D = RG_PF_D * CELLS <= 256 ? RG_PF_D : 256 / CELLS; };  // <= 32 KiB static smem
 
+// shared-memory offset (ints) of cell k of `lane` in ring slot `slot`: [slot][q][lane][4] for
+// CELLS % 4 == 0, [slot][lane][2] for 2-cell lanes (64-bit accesses, also conflict free)
+template <int CELLS>
+__device__ __forceinline__ int pf_off(int slot, int lane, int k) {
+    if constexpr (CELLS % 4 == 0) return (slot * (CELLS / 4) * 32 + lane) * 4 + (k / 4) * 128 + (k % 4);
+    else return (slot * 32 + lane) * CELLS + k;
+}
+
 template <int CELLS, bool EC>
 __device__ __forceinline__ void pf_issue(int32_t* ring, const int32_t* __restrict__ wall, int row, int C,
                                          int col0, int lane, int slot) {
     // layout [slot][q][lane][4]: for a fixed 16-byte chunk q the 32 lanes are contiguous, so the
     // 128-bit shared stores and loads are bank-conflict free for any CELLS
-    int32_t* dst = ring + (slot * (CELLS / 4) * 32 + lane) * 4;
+    int32_t* dst = ring + pf_off<CELLS>(slot, lane, 0);
     const int32_t* src = wall + (size_t)row * C;
-    if (!EC) {
+    if (!EC && CELLS == 2) {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+                     "l"(src + col0));
+    } else if (!EC) {
 #pragma unroll
         for (int q = 0; q < CELLS / 4; ++q)
             asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + q * 128)),
@@ -164,7 +175,7 @@ __device__ __forceinline__ void pf_issue(int32_t* ring, const int32_t* __restric
         for (int k = 0; k < CELLS; ++k) {
             const int c = col0 + k;
             const bool ok = c >= 0 && c < C;
-            asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(dst + (k / 4) * 128 + (k % 4))),
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"((uint32_t)__cvta_generic_to_shared(ring + pf_off<CELLS>(slot, lane, k))),
                          "l"(ok ? src + c : wall), "r"(ok ? 4 : 0));
         }
     }
@@ -183,7 +194,10 @@ __device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, c
     cudaGridDependencySynchronize();  // PDL: prev_in is produced by the previous launch
 #endif
     int32_t v[CELLS];
-    if (!EC) {
+    if (!EC && CELLS == 2) {
+        const int2 t = *reinterpret_cast<const int2*>(prev_in + col0);
+        v[0] = t.x; v[1 % CELLS] = t.y;
+    } else if (!EC) {
 #pragma unroll
         for (int q = 0; q < CELLS / 4; ++q) {
             const int4 t = *reinterpret_cast<const int4*>(prev_in + col0 + 4 * q);
@@ -196,7 +210,11 @@ __device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, c
     for (int i = 0; i < h; ++i) {
         asm volatile("cp.async.wait_group %0;\n" ::"n"(PfRing<CELLS>::D - 2));
         int32_t w[CELLS];
-        const int32_t* src = ring + ((i & (PfRing<CELLS>::D - 1)) * (CELLS / 4) * 32 + lane) * 4;
+        const int32_t* src = ring + pf_off<CELLS>(i & (PfRing<CELLS>::D - 1), lane, 0);
+        if constexpr (CELLS == 2) {
+            const int2 t = *reinterpret_cast<const int2*>(src);
+            w[0] = t.x; w[1 % CELLS] = t.y;
+        }
 #pragma unroll
         for (int q = 0; q < CELLS / 4; ++q) {
             const int4 t = reinterpret_cast<const int4*>(src)[q * 32];
@@ -270,6 +288,7 @@ static const Variant* find(int cells, int mode) {
 
 struct BandVariant { int cells; PfFn fn; const char* key; };
 static const BandVariant kBand[] = {
+    {2, pf_band<2>, "void rg::pf_band<2>"},
     {4, pf_band<4>, "void rg::pf_band<4>"},   {8, pf_band<8>, "void rg::pf_band<8>"},
     {16, pf_band<16>, "void rg::pf_band<16>"}, {32, pf_band<32>, "void rg::pf_band<32>"},
 };

@@ -8,7 +8,8 @@ import os
 import subprocess
 import sys
 
-GRANS = [(c, 1, 1, 1, h, 1, 2) for c in (4, 8) for h in (12, 16, 20, 24, 28)] + \
+GRANS = [(4, 1, 1, 1, 20, 1, 2)] + [(2, 1, 1, 1, h, 1, 2) for h in (4, 8, 12, 16, 20)] + \
+        [(c, 1, 1, 1, h, 1, 2) for c in (4, 8) for h in (12, 16, 24, 28)] + \
         [(16, 1, 1, 1, h, 1, 2) for h in (33, 50, 99)]
 
 CHILD = r"""
