@@ -50,7 +50,9 @@ typedef enum {
     RODINIA_E_SMEM = -3,           /* variant needs more shared memory per CTA than the device
                                       offers (early pruning)                    */
     RODINIA_E_FILTERED = -4,       /* variant rejected by the compile-time ptxas filter: new
-                                      spills or < 1 CTA/SM                     */
+                                      spills or < 1 CTA/SM.  Returned by every
+                                      entry point for an explicitly requested pruned
+                                      instantiation unless flags has RODINIA_FORCE          */
     RODINIA_E_NOT_BUILT = -5,      /* factor combination not instantiated in this build       */
     RODINIA_E_DEGENERATE = -6,     /* srad: ROI mean == 0, q0sqr undefined                     */
     RODINIA_E_NODEV = -7,          /* no CUDA device / driver                                  */
@@ -78,6 +80,9 @@ typedef enum {
  *                      divide the original tile).
  *                      bit1 RODINIA_STREAM -- use the streaming temporal-blocking family
  *                      (hotspot).
+ *                      bit2 RODINIA_FORCE -- run the instantiation even if the compile-time
+ *                      ptxas filter pruned it (new spills / 0 CTAs per SM);
+ *                      without it such a call returns RODINIA_E_FILTERED before any launch.
  *                      bits 8..15 RODINIA_OCC(n) -- register budget of the instantiation:
  *                      target n resident CTAs per SM (launch bounds => <= 65536/(threads*n)
  *                      registers per thread); 0 = the family's preferred instantiation.  This
@@ -95,6 +100,7 @@ typedef struct {
 
 #define RODINIA_FAITHFUL 1
 #define RODINIA_STREAM 2
+#define RODINIA_FORCE 4
 #define RODINIA_OCC(n) (((n) & 0xff) << 8)
 #define RODINIA_OCC_OF(flags) (((flags) >> 8) & 0xff)
 

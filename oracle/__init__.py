@@ -25,8 +25,10 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "rodinia_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
 _lock = threading.Lock()
 _lib = None
+_threads = 1
 
 OK = 0
 EINVAL = -1
@@ -36,20 +38,43 @@ ENOMEM = -10
 _CFLAGS = ["-O2", "-std=c99", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared"]
 
 
-def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc (no fast-math, no FMA contraction)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *_CFLAGS, "-o", tmp, _SRC, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+def build(force: bool = False, omp: bool = False) -> str:
+    """Compile liboracle.so with gcc (no fast-math, no FMA contraction); with omp=True the
+    OpenMP build liboracle_omp.so (same source, per-cell stencil loops threaded, identical bits).
+    """
+    lib = _LIB_OMP if omp else _LIB
+    if force or not os.path.exists(lib) or os.path.getmtime(lib) < os.path.getmtime(_SRC):
+        tmp = lib + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *_CFLAGS, *(["-fopenmp"] if omp else []), "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, lib)
+    return lib
+
+
+def set_threads(n: int) -> int:
+    """Select the single-threaded build (n == 1, the default) or the OpenMP build with n threads
+    (n == 0: all host cores, os.cpu_count()).  Returns the thread count in effect.  Results are
+    bitwise identical either way (only independent per-cell loops are threaded)."""
+    global _lib, _threads
+    n = os.cpu_count() or 1 if n == 0 else int(n)
+    with _lock:
+        if n != _threads or _lib is None:
+            _lib = None
+            _threads = n
+    lib = _load()
+    return int(lib.oracle_set_threads(n))
+
+
+def threads() -> int:
+    return _threads
 
 
 def _load():
     global _lib
     with _lock:
         if _lib is None:
-            lib = ctypes.CDLL(build())
+            lib = ctypes.CDLL(build(omp=_threads > 1))
+            lib.oracle_set_threads.argtypes = [ctypes.c_int]
+            lib.oracle_set_threads.restype = ctypes.c_int
             d, l, i = ctypes.c_double, ctypes.c_long, ctypes.c_int
             pd = ctypes.POINTER(ctypes.c_double)
             pi32 = ctypes.POINTER(ctypes.c_int32)

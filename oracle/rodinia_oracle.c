@@ -19,7 +19,11 @@
  * Every reading where the paper is silent is listed in DESIGN.md §3 ("Readings").
  *
  * Build: gcc -O2 -std=c99 -ffp-contract=off -fPIC -shared (no fast-math).
- * Single-threaded, deterministic.
+ * Single-threaded, deterministic.  A second build with -fopenmp (liboracle_omp.so) spreads the
+ * independent per-cell loops of the stencil steps (hotspot, srad passes 1/2, pathfinder's row,
+ * hotspot3D) over threads for the CPU baseline on the GPU box's cores; every
+ * cell's arithmetic and every reduction (the ROI sums, lud) are unchanged and sequential, so
+ * both builds return identical bits.
  */
 #include <math.h>
 #include <stdint.h>
@@ -30,6 +34,25 @@
 #define ORACLE_EINVAL (-1)
 #define ORACLE_EDEGENERATE (-6)
 #define ORACLE_ENOMEM (-10)
+
+#ifdef _OPENMP
+#include <omp.h>
+#define ORACLE_PAR _Pragma("omp parallel for schedule(static)")
+#else
+#define ORACLE_PAR
+#endif
+
+/* Threads used by the per-cell loops (OpenMP build); returns the count in effect (1 without
+ * OpenMP). */
+int oracle_set_threads(int n) {
+#ifdef _OPENMP
+    if (n >= 1) omp_set_num_threads(n);
+    return omp_get_max_threads();
+#else
+    (void)n;
+    return 1;
+#endif
+}
 
 static long lmin(long a, long b) { return a < b ? a : b; }
 static long lmax(long a, long b) { return a > b ? a : b; }
@@ -74,6 +97,7 @@ int oracle_hotspot_coeffs_rodinia(long rows, long cols, double chip_w, double ch
  */
 static void hotspot_step(const double* t, const double* p, double* out, long R, long C,
                          double k, double rx, double ry, double rz, double amb) {
+    ORACLE_PAR
     for (long i = 0; i < R; ++i) {
         long in = lmax(i - 1, 0), is = lmin(i + 1, R - 1);
         for (long j = 0; j < C; ++j) {
@@ -146,6 +170,7 @@ int oracle_srad_q0sqr(const double* J, long R, long C, long r1, long r2, long c1
  * Writes c (R*C).  The four differences are recomputed by pass 2 from the same J. */
 int oracle_srad_coeff(const double* J, long R, long C, double q0sqr, double* cout) {
     if (!J || !cout || R < 1 || C < 1) return ORACLE_EINVAL;
+    ORACLE_PAR
     for (long i = 0; i < R; ++i) {
         long in = lmax(i - 1, 0), is = lmin(i + 1, R - 1);
         for (long j = 0; j < C; ++j) {
@@ -174,6 +199,7 @@ int oracle_srad_coeff(const double* J, long R, long C, double q0sqr, double* cou
  * jold and jnew must not alias. */
 static void srad_update(const double* jold, const double* c, double* jnew, long R, long C,
                         double lambda) {
+    ORACLE_PAR
     for (long i = 0; i < R; ++i) {
         long in = lmax(i - 1, 0), is = lmin(i + 1, R - 1);
         for (long j = 0; j < C; ++j) {
@@ -233,6 +259,7 @@ int oracle_pathfinder(const int32_t* wall, long R, long C, int32_t* result) {
     if (!prev || !next) { free(prev); free(next); return ORACLE_ENOMEM; }
     memcpy(prev, wall, (size_t)C * sizeof(int32_t));
     for (long r = 1; r < R; ++r) {
+        ORACLE_PAR
         for (long j = 0; j < C; ++j) {
             int32_t m = prev[j];
             if (j > 0 && prev[j - 1] < m) m = prev[j - 1];
@@ -332,6 +359,7 @@ int oracle_hotspot3d(const double* t0, const double* p, double* out, long nx, lo
     if (!cur || !nxt) { free(cur); free(nxt); return ORACLE_ENOMEM; }
     memcpy(cur, t0, n * sizeof(double));
     for (int it = 0; it < iters; ++it) {
+        ORACLE_PAR
         for (long z = 0; z < nz; ++z)
             for (long y = 0; y < ny; ++y)
                 for (long x = 0; x < nx; ++x) {

@@ -40,6 +40,7 @@ RODINIA_E_PRUNED = -11
 
 RODINIA_FAITHFUL = 1
 RODINIA_STREAM = 2
+RODINIA_FORCE = 4  # run an instantiation the compile-time filter pruned (else RODINIA_E_FILTERED)
 
 RODINIA_HOTSPOT, RODINIA_SRAD, RODINIA_PATHFINDER, RODINIA_LUD, RODINIA_HOTSPOT3D = 0, 1, 2, 3, 4
 KERNELS = {"hotspot": 0, "srad": 1, "pathfinder": 2, "lud": 3, "hotspot3d": 4}

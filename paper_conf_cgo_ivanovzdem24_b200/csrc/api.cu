@@ -399,6 +399,7 @@ HostStage& host_stage() {
     static HostStage hs;
     return hs;
 }
+std::mutex& host_mutex() { return host_stage().mu; }
 rodinia_status host_buffer(int i, size_t bytes, void** out) {
     HostStage& hs = host_stage();
     int dev = 0;

@@ -483,7 +483,9 @@ rodinia_status check(const rodinia_granularity& g, int64_t R, int64_t C,
         if (!*sv)
             return set_error(RODINIA_E_NOT_BUILT, "hotspot: stream variant %s not instantiated", gran_str(g).c_str());
     }
-    return RODINIA_OK;
+    // compile-time filter at the boundary
+    return *dv ? boundary_filter(RODINIA_HOTSPOT, (*dv)->key, (16 / (*dv)->tx) * (16 / (*dv)->ty), 0, g.flags)
+               : boundary_filter(RODINIA_HOTSPOT, (*sv)->key, 32, 0, g.flags);
 }
 
 static void launch_direct(const DirectVariant* dv, int bx, int by, const float* tin, const float* p,

@@ -274,7 +274,8 @@ rodinia_status check(const rodinia_granularity& g, int64_t ny, const Variant** o
     }
     *out = find(g.thread_x, g.thread_y, g.index_mode, plane);
     if (!*out) return set_error(RODINIA_E_NOT_BUILT, "hotspot3d: variant %s not instantiated", gran_str(g).c_str());
-    return RODINIA_OK;
+    return boundary_filter(RODINIA_HOTSPOT3D, (*out)->key, plane ? 256 : (64 / g.thread_x) * (4 / g.thread_y), 0,
+                           g.flags);  // compile-time filter at the boundary
 }
 
 int num_variants() { return (int)(sizeof(kVariants) / sizeof(kVariants[0]) + sizeof(kPlane) / sizeof(kPlane[0])); }
@@ -401,6 +402,7 @@ extern "C" rodinia_status rodinia_hotspot3d_host(const float* tin, const float* 
     RG_TRY(device_info(&di));
     const size_t bytes = (size_t)nx * ny * nz * 4;
     void *dt, *dp, *dout;
+    std::lock_guard<std::mutex> lk(host_mutex());  // cached buffers: whole H2D/solve/D2H
     RG_TRY(host_buffer(0, bytes, &dt));
     RG_TRY(host_buffer(1, bytes, &dp));
     RG_TRY(host_buffer(2, bytes, &dout));

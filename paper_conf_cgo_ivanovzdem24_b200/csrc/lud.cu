@@ -467,7 +467,7 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
         pl->by = g.block_y;  // rows per CTA in 16-row tiles
         pl->smem = (size_t)16 * g.block_y * panel * sizeof(float);
         if (pl->smem > 227 * 1024) return set_error(RODINIA_E_SMEM, "lud: stream chunk needs %zu B shared memory", pl->smem);
-        return RODINIA_OK;
+        return boundary_filter(RODINIA_LUD, pl->sv->key, 256, (int)pl->smem, g.flags);
     }
     if (panel % g.thread_x || panel % g.thread_y)
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "lud: thread factors must divide the %dx%d tile (PAPER.md:237)", panel, panel);
@@ -480,7 +480,8 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
     if (pl->smem > 227 * 1024)
         return set_error(RODINIA_E_SMEM, "lud: block factor (%d,%d) needs %zu B shared memory > 227 KB (PAPER.md:251)",
                          g.block_x, g.block_y, pl->smem);
-    return RODINIA_OK;
+    return boundary_filter(RODINIA_LUD, pl->v->key, (panel / g.thread_x) * (panel / g.thread_y), (int)pl->smem,
+                           g.flags);  // compile-time filter at the boundary
 }
 
 static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
@@ -504,8 +505,17 @@ static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
     }
 }
 
+// One captured factorisation per (device, n, plan).  The matrix pointer reaches the kernels
+// through a device slot written by the graph's own root node (lud_set_slot), whose argument is
+// replaced with cudaGraphExecKernelNodeSetParams before every launch.  Launches of one graph
+// exec are ordered after each other whatever their streams, and a parameter update only affects
+// later launches, so concurrent calls with the same n on different streams each factor their own
+// matrix (the slot and the panel-128 operand images are only touched inside the graph).
 struct GraphEntry {
+    cudaGraph_t graph = nullptr;      // kept alive: `root` must stay a node of it
     cudaGraphExec_t exec = nullptr;
+    cudaGraphNode_t root = nullptr;   // the lud_set_slot kernel node
+    cudaKernelNodeParams rootp = {};
     float** slot = nullptr;
     float* img = nullptr;   // panel-128 path: the two tensor-core operand images
     int launches = 0;
@@ -523,28 +533,43 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
     GraphEntry& ge = g_graphs[key];
     const int m = (n + pl.p - 1) / pl.p;
     if (!ge.exec) {
-        RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
+        if (!ge.slot) RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
         const void* ifn = pl.tc ? (const void*)tc::lud_tc_update2
                                 : pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
-        if (pl.tc) RG_CUDA(cudaMalloc(&ge.img, 2 * tc::img_floats(n) * sizeof(float)));
+        if (pl.tc && !ge.img) RG_CUDA(cudaMalloc(&ge.img, 2 * tc::img_floats(n) * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
         cudaStream_t cs;
         RG_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
         cudaGraph_t graph;
         RG_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+        lud_set_slot<<<1, 1, 0, cs>>>(ge.slot, a);  // root node; argument replaced per launch
         int nl = 3 * m - 2;
         if (pl.tc) nl = tc::launch_all(ge.slot, n, ge.img, ge.img + tc::img_floats(n), cs);
         else launch_all(pl, ge.slot, n, cs);
         cudaError_t e = cudaStreamEndCapture(cs, &graph);
         cudaStreamDestroy(cs);
         if (e != cudaSuccess) return cuda_error(e, "lud graph capture", __FILE__, __LINE__);
-        e = cudaGraphInstantiate(&ge.exec, graph, 0);
-        cudaGraphDestroy(graph);
-        if (e != cudaSuccess) { ge.exec = nullptr; return cuda_error(e, "lud graph instantiate", __FILE__, __LINE__); }
+        size_t nroot = 1;
+        cudaGraphNode_t root = nullptr;
+        e = cudaGraphGetRootNodes(graph, &root, &nroot);
+        if (e == cudaSuccess && nroot == 1) e = cudaGraphKernelNodeGetParams(root, &ge.rootp);
+        else if (e == cudaSuccess) e = cudaErrorInvalidValue;
+        if (e == cudaSuccess) e = cudaGraphInstantiate(&ge.exec, graph, 0);
+        if (e != cudaSuccess) {
+            ge.exec = nullptr;
+            cudaGraphDestroy(graph);
+            return cuda_error(e, "lud graph instantiate", __FILE__, __LINE__);
+        }
+        ge.graph = graph;
+        ge.root = root;
         ge.launches = nl;
     }
-    lud_set_slot<<<1, 1, 0, s>>>(ge.slot, a);
+    void* args[2] = {(void*)&ge.slot, (void*)&a};
+    cudaKernelNodeParams kp = ge.rootp;
+    kp.kernelParams = args;
+    kp.extra = nullptr;
+    RG_CUDA(cudaGraphExecKernelNodeSetParams(ge.exec, ge.root, &kp));
     RG_CUDA(cudaGraphLaunch(ge.exec, s));
     count_launch(ge.launches + 1);
     return RODINIA_OK;
@@ -697,7 +722,22 @@ extern "C" rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const 
     RG_TRY(lud::plan(gg, panel, &pl));
     DeviceInfo di;
     RG_TRY(device_info(&di));
-    return lud::run(a, (int)n, pl, (cudaStream_t)stream);
+    cudaStream_t s = (cudaStream_t)stream;
+    if ((reinterpret_cast<uintptr_t>(a) & 15) == 0) return lud::run(a, (int)n, pl, s);
+    // The kernels' 128-bit accesses (and the panel-128 bulk reduce-add) need a 16-byte aligned
+    // matrix; an offset view is factored in an aligned stream-ordered copy (same kernels, same
+    // bits) and copied back.
+    const size_t bytes = (size_t)n * n * sizeof(float);
+    float* t = nullptr;
+    RG_TRY(scratch_alloc((void**)&t, bytes, s));
+    rodinia_status st = RODINIA_OK;
+    if (cudaMemcpyAsync(t, a, bytes, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        st = cuda_error(cudaGetLastError(), "lud aligned copy", __FILE__, __LINE__);
+    if (st == RODINIA_OK) st = lud::run(t, (int)n, pl, s);
+    if (st == RODINIA_OK && cudaMemcpyAsync(a, t, bytes, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        st = cuda_error(cudaGetLastError(), "lud aligned copy", __FILE__, __LINE__);
+    scratch_free(t, s);
+    return st;
 }
 
 extern "C" rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
@@ -706,6 +746,7 @@ extern "C" rodinia_status rodinia_lud_host(float* a, int64_t n, int32_t panel, c
     DeviceInfo di;
     RG_TRY(device_info(&di));
     void* da;
+    std::lock_guard<std::mutex> lk(host_mutex());  // cached buffers: whole H2D/solve/D2H
     RG_TRY(host_buffer(0, (size_t)n * n * 4, &da));
     cudaStream_t s = (cudaStream_t)stream;
     RG_CUDA(cudaMemcpyAsync(da, a, (size_t)n * n * 4, cudaMemcpyHostToDevice, s));

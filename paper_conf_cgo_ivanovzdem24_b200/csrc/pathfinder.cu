@@ -32,7 +32,8 @@ namespace rg {
 template <int CELLS, int MODE>
 __global__ void __launch_bounds__(256)
     pf_pyramid(const int32_t* __restrict__ wall, const int32_t* __restrict__ prev_in,
-               int32_t* __restrict__ next_out, int R, int C, int r0, int h, int band_out) {
+               int32_t* __restrict__ next_out, int R, int C, int r0, int h, int band_out, int vec_ok) {
+    (void)vec_ok;  // scalar accesses only
     // staged band: columns [b0 - h, b0 - h + NT*CELLS), outputs [b0, b0 + band_out)
     extern __shared__ int32_t pf_edges[];  // [2][nwarps][2]
     const int nt = blockDim.x;
@@ -253,14 +254,16 @@ __device__ __forceinline__ void pf_band_body(const int32_t* __restrict__ wall, c
 template <int CELLS>
 __global__ void __launch_bounds__(32)
     pf_band(const int32_t* __restrict__ wall, const int32_t* __restrict__ prev_in, int32_t* __restrict__ next_out,
-            int R, int C, int r0, int h, int band_out) {
+            int R, int C, int r0, int h, int band_out, int vec_ok) {
     __shared__ __align__(16) int32_t ring[PfRing<CELLS>::D * 32 * CELLS];
     const int lane = threadIdx.x;
     const int halo = (h + 3) & ~3;
     const int b0 = blockIdx.x * band_out;
     const int s0 = b0 - halo;
     const int col0 = s0 + lane * CELLS;
-    const bool ec = ((C & 3) != 0) || s0 < 0 || s0 + 32 * CELLS > C;
+    // vector (int2 / int4, cp.async 8/16 B) accesses need C % 4 == 0 and 16-byte aligned wall,
+    // prev_in and next_out (vec_ok, checked on the host); otherwise the scalar edge path
+    const bool ec = !vec_ok || ((C & 3) != 0) || s0 < 0 || s0 + 32 * CELLS > C;
     if (ec) pf_band_body<CELLS, true>(wall, prev_in, next_out, ring, C, r0, h, b0, band_out, col0, lane);
     else pf_band_body<CELLS, false>(wall, prev_in, next_out, ring, C, r0, h, b0, band_out, col0, lane);
     (void)R;
@@ -268,7 +271,7 @@ __global__ void __launch_bounds__(32)
 
 namespace pathfinder {
 
-typedef void (*PfFn)(const int32_t*, const int32_t*, int32_t*, int, int, int, int, int);
+typedef void (*PfFn)(const int32_t*, const int32_t*, int32_t*, int, int, int, int, int, int);
 struct Variant { int cells, mode; PfFn fn; const char* key; };
 
 #define RG_PF(N, M) {N, M, pf_pyramid<N, M>, "void rg::pf_pyramid<" #N ", " #M ">"}
@@ -325,7 +328,7 @@ rodinia_status plan(const rodinia_granularity& g, int64_t R, int64_t C, Plan* p)
             return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: pyramid height %d too large for a %d-column band",
                              p->h, 32 * cells);
         p->launches = steps > 0 ? (int)((steps + p->h - 1) / p->h) : 0;
-        return RODINIA_OK;
+        return boundary_filter(RODINIA_PATHFINDER, p->band->key, 32, 0, g.flags);
     }
     if ((g.flags & RODINIA_FAITHFUL) && (256 % t != 0))
         return set_error(RODINIA_E_ILLEGAL_FACTOR, "pathfinder: thread factor %d does not divide the "
@@ -345,7 +348,7 @@ rodinia_status plan(const rodinia_granularity& g, int64_t R, int64_t C, Plan* p)
                                                    "band", p->h, threads * cells);
     p->launches = steps > 0 ? (int)((steps + p->h - 1) / p->h) : 0;
     (void)C;
-    return RODINIA_OK;
+    return boundary_filter(RODINIA_PATHFINDER, p->v->key, threads, 0, g.flags);
 }
 
 rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R, int C, const Plan& p,
@@ -360,6 +363,8 @@ rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R
     PfFn fn = p.band ? p.band->fn : p.v->fn;
     const int32_t* src = wall;  // row 0 of the wall is the initial cost
     int r0 = 0;
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(wall) | reinterpret_cast<uintptr_t>(result) |
+                         reinterpret_cast<uintptr_t>(scratch)) % 16) == 0;
     for (int l = 0; l < p.launches; ++l) {
         const int h = std::min(p.h, R - 1 - r0);
         int32_t* dst = ((p.launches - 1 - l) % 2 == 0) ? result : scratch;
@@ -373,7 +378,7 @@ rodinia_status run(const int32_t* wall, int32_t* result, int32_t* scratch, int R
         attr[0].val.programmaticStreamSerializationAllowed = 1;
         cfg.attrs = attr;
         cfg.numAttrs = l > 0 ? 1 : 0;
-        RG_CUDA(cudaLaunchKernelEx(&cfg, fn, wall, (const int32_t*)src, dst, R, C, r0, h, p.band_out));
+        RG_CUDA(cudaLaunchKernelEx(&cfg, fn, wall, (const int32_t*)src, dst, R, C, r0, h, p.band_out, vec_ok));
         count_launch();
         src = dst;
         r0 += h;
@@ -539,6 +544,7 @@ extern "C" rodinia_status rodinia_pathfinder_host(const int32_t* wall, int64_t R
     DeviceInfo di;
     RG_TRY(device_info(&di));
     void *dw, *dr;
+    std::lock_guard<std::mutex> lk(host_mutex());  // cached buffers: whole H2D/solve/D2H
     RG_TRY(host_buffer(0, (size_t)R * C * 4, &dw));
     RG_TRY(host_buffer(1, (size_t)C * 4, &dr));
     cudaStream_t s = (cudaStream_t)stream;

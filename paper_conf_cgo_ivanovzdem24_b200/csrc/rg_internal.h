@@ -5,6 +5,7 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -62,6 +63,10 @@ const PtxasStats* find_stats(const char* key);  // nullptr if unknown
 // `base_spill` is the spill bytes of the family's uncoarsened kernel (new spills are pruned).
 rodinia_status filter_decision(const PtxasStats* st, int threads, int smem_bytes, int base_spill);
 
+// The filter applied at the boundary to an explicitly requested instantiation: RODINIA_OK, or
+// RODINIA_E_FILTERED / RODINIA_E_SMEM with a message, unless flags & RODINIA_FORCE.
+rodinia_status boundary_filter(rodinia_kernel k, const char* key, int threads, int dyn_smem, int flags);
+
 // Occupancy query (CTAs / SM) of a kernel at block size and dynamic smem; 0 on failure.
 int ctas_per_sm(const void* func, int threads, size_t dyn_smem);
 
@@ -81,8 +86,10 @@ std::string gran_str(const rodinia_granularity& g);
 // Default granularity per workload when neither the caller nor the tune cache chooses one.
 rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p);
 
-// Cached device buffers of the *_host entry points (index 0..2), grown on demand.
+// Cached device buffers of the *_host entry points (index 0..2), grown on demand.  The caller
+// holds host_mutex() for the whole H2D / solve / D2H / sync sequence that uses them.
 rodinia_status host_buffer(int i, size_t bytes, void** out);
+std::mutex& host_mutex();
 
 // ------------------------------------------------------------------ pre-pruning (tune.cu, model.cu)
 // Model estimate of one call at row.g (rodinia_model_ms); -1 when the workload is not modelled.

@@ -91,6 +91,24 @@ static int family_base_spill(rodinia_kernel k) {
     return st ? st->spill_stores + st->spill_loads : 0;
 }
 
+// The compile-time filter at the boundary: an explicitly requested
+// instantiation the ptxas filter prunes is refused with RODINIA_E_FILTERED (host-only, before
+// any launch) unless the caller sets RODINIA_FORCE.  Same decision as rodinia_variants().
+rodinia_status boundary_filter(rodinia_kernel k, const char* key, int threads, int dyn_smem, int flags) {
+    if (flags & RODINIA_FORCE) return RODINIA_OK;
+    static int base[5] = {-1, -1, -1, -1, -1};
+    const int ki = (int)k;
+    if (ki < 0 || ki >= 5) return RODINIA_OK;
+    if (base[ki] < 0) base[ki] = family_base_spill(k);
+    const PtxasStats* st = find_stats(key);
+    const rodinia_status s = filter_decision(st, threads, dyn_smem, base[ki]);
+    if (s == RODINIA_OK) return RODINIA_OK;
+    return set_error(s, "%s is pruned by the compile-time filter (%d registers, %d B spill stores + %d B "
+                        "loads, %d B shared memory, %d threads; PAPER.md:267); set RODINIA_FORCE to run it",
+                     key, st ? st->regs : -1, st ? st->spill_stores : -1, st ? st->spill_loads : -1,
+                     (st ? st->smem : 0) + dyn_smem, threads);
+}
+
 rodinia_granularity default_gran(rodinia_kernel k, const rodinia_problem& p) {
     switch (k) {
         case RODINIA_HOTSPOT:

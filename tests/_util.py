@@ -42,3 +42,30 @@ def rel_err(a, b):
     a = np.asarray(a, dtype=np.float64)
     b = np.asarray(b, dtype=np.float64)
     return np.max(np.abs(a - b) / np.maximum(np.abs(b), 1e-30)) if a.size else 0.0
+
+
+def hotspot_window_block(T, P, i0, j0, h, w, iters, coef):
+    """Oracle values (fp64) of the h x w output block at (i0, j0) after `iters` steps: the plain
+    oracle on the block grown by the cone radius iters + 1 (clamped to the grid, where the
+    window then coincides with the real boundary)."""
+    R, C = T.shape
+    r = iters + 1
+    a0, a1 = max(0, i0 - r), min(R, i0 + h + r)
+    b0, b1 = max(0, j0 - r), min(C, j0 + w + r)
+    out = oracle.hotspot(T[a0:a1, b0:b1], P[a0:a1, b0:b1], iters, coef["k"], coef["rx"],
+                         coef["ry"], coef["rz"], coef["amb"])
+    return out[i0 - a0:i0 - a0 + h, j0 - b0:j0 - b0 + w]
+
+
+def srad_window_block(J, i0, j0, h, w, niter, q0_seq, lam):
+    """Oracle values of the h x w srad output block at (i0, j0) after niter iterations, given the
+    full grid's q0sqr sequence; window = block grown by 2*niter + 2 on every side (the cone
+    reaches niter rows/cols toward lower and 2*niter toward higher indices)."""
+    R, C = J.shape
+    m = 2 * niter + 2
+    a0, a1 = max(0, i0 - m), min(R, i0 + h + m)
+    b0, b1 = max(0, j0 - m), min(C, j0 + w + m)
+    x = np.asarray(J[a0:a1, b0:b1], dtype=np.float64)
+    for t in range(niter):
+        x = oracle.srad_step(x, q0_seq[t], lam)
+    return x[i0 - a0:i0 - a0 + h, j0 - b0:j0 - b0 + w]

@@ -130,3 +130,49 @@ def test_hotspot_host_batch_argument_validation_without_device():
     assert rg.lib.rodinia_hotspot_host_batch(null3, ok, ok, 1, 8, 8, 1, None, None, None) == rg.RODINIA_E_INVALID
     assert rg.lib.rodinia_hotspot_host_batch(ok, ok, ok, 1, 0, 8, 1, None, None, None) == rg.RODINIA_E_INVALID
     assert rg.lib.rodinia_hotspot_host_batch(None, None, None, 0, 8, 8, 1, None, None, None) == rg.RODINIA_OK
+
+
+def _nodev_or_ok():
+    import torch
+    return rg.RODINIA_OK if torch.cuda.is_available() else rg.RODINIA_E_NODEV
+
+
+def test_filter_enforced_at_the_boundary():
+    # An explicit call naming an instantiation the compile-time ptxas filter pruned (new spills,
+    # PAPER.md:267) is refused before any CUDA call; RODINIA_FORCE runs it anyway.  hotspot:
+    # hs_stream<4, 4, 16> (V = 4, H = 4, OCC 16 -> <= 128 registers) spills in this build.
+    S, F = rg.RODINIA_STREAM, rg.RODINIA_FORCE
+    spilling = (4, 1, 1, 4, 4, 1, S | (16 << 8))
+    rows = {r["g"]: r for r in rg.rodinia_variants("hotspot")}
+    assert rows[spilling]["status"] == rg.RODINIA_E_FILTERED and rows[spilling]["spill_bytes"] > 0
+    assert _hs(R=64, C=256, g=spilling) == rg.RODINIA_E_FILTERED
+    assert "RODINIA_FORCE" in rg.last_error()
+    if _nodev_or_ok() == rg.RODINIA_E_NODEV:  # past the filter the call needs a device
+        assert _hs(R=64, C=256, g=spilling[:6] + (spilling[6] | F,)) == rg.RODINIA_E_NODEV
+    # every pruned hotspot instantiation is refused, every surviving one passes the filter
+    for g, r in rows.items():
+        st = _hs(R=64, C=256, g=g)
+        if r["status"] == rg.RODINIA_E_FILTERED:
+            assert st == rg.RODINIA_E_FILTERED, g
+        else:
+            assert st != rg.RODINIA_E_FILTERED, g
+
+
+def test_filter_enforced_lud_and_others():
+    # lud: the pruned internal instantiations (panel 16 or 32; the listing's granularity does not
+    # carry the panel width, so one of the two must refuse it)
+    lud = lambda g, panel: rg.lib.rodinia_lud(ctypes.c_void_p(16), 256, panel, rg._g(g), None)
+    pruned = [r["g"] for r in rg.rodinia_variants("lud") if r["status"] == rg.RODINIA_E_FILTERED]
+    assert pruned
+    for g in pruned:
+        sts = {lud(g, 16), lud(g, 32)}
+        assert rg.RODINIA_E_FILTERED in sts, g
+        forced = g[:6] + (g[6] | rg.RODINIA_FORCE,)
+        assert rg.RODINIA_E_FILTERED not in {lud(forced, 16), lud(forced, 32)}, g
+    # srad / pathfinder / hotspot3d: nothing is pruned in this build; surviving variants pass
+    for k in ("srad", "pathfinder", "hotspot3d"):
+        for r in rg.rodinia_variants(k):
+            assert r["status"] in (rg.RODINIA_OK, rg.RODINIA_E_FILTERED)
+    sr = rg.lib.rodinia_srad(ctypes.c_void_p(16), 64, 64, 0, 9, 0, 9, ctypes.c_float(0.5), 2,
+                             rg._g((4, 1, 1, 2, 1, 1, rg.RODINIA_STREAM)), None)
+    assert sr == _nodev_or_ok()

@@ -9,7 +9,7 @@ import pytest
 
 import oracle
 import synth
-from tests._util import hotspot_window_value, rel_err
+from tests._util import hotspot_window_block, rel_err
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
@@ -108,24 +108,34 @@ def test_pins_on_gpu(rg):
     assert rel_err(out, T) <= 1e-6
 
 
-def test_full_size_sampled_vs_oracle(rg):
-    # BASELINE configs[2] at full size (16384^2, 1000 iterations, 512-grid coefficients) in
-    # the default (bench) launch configuration, sampled cells checked against the windowed
-    # oracle; the whole output is compared bitwise with the uncoarsened variant over 24 steps.
-    N = 16384
+def test_full_size_windows_vs_oracle(rg):
+    # BASELINE configs[2] at full size (16384^2, 1000 iterations, 512-grid coefficients) in the
+    # launch configuration bench.py times: the TDO winner of the same rodinia_tune call (it is
+    # also what a NULL granularity resolves to afterwards).  Three 64 x 64 output windows -- the
+    # grid corner, a bottom-edge strip and the interior -- are compared elementwise with the
+    # windowed fp64 oracle (cone radius 1001, OpenMP build over the host cores); the whole
+    # output is compared bitwise with the uncoarsened variant over 24 steps.
+    N, n = 16384, 1000
     T, P = synth.hotspot_inputs(N, N)
     coef = _coef32(oracle.hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6))
+    g, _ = rg.rodinia_tune("hotspot", N, N, n, nranks=1, reps=2)
+    assert rg.rodinia_resolve("hotspot", N, N, n).astuple() == g.astuple()
     t = torch.from_numpy(T).cuda()
     p = torch.from_numpy(P).cuda()
     c = rg.coeffs(coef["k"], coef["rx"], coef["ry"], coef["rz"], coef["amb"])
-    a = rg.rodinia_hotspot(t, p, 24, coeffs=c, g=None)
+    a = rg.rodinia_hotspot(t, p, 24, coeffs=c, g=g)
     b = rg.rodinia_hotspot(t, p, 24, coeffs=c, g=UNC)
-    assert torch.equal(a, b)
-    out = rg.rodinia_hotspot(t, p, 1000, coeffs=c, g=None).cpu().numpy()
-    for (i, j) in [(0, 0), (N - 1, 5), (8191, 12000)]:
-        ref = hotspot_window_value(T, P, i, j, 1000, coef)
-        assert abs(out[i, j] - ref) <= TOL * abs(ref), (i, j, out[i, j], ref)
+    assert torch.equal(a, b), g.astuple()
+    out = rg.rodinia_hotspot(t, p, n, coeffs=c, g=None).cpu().numpy()
     assert np.isfinite(out).all()
+    oracle.set_threads(0)
+    try:
+        for (i0, j0) in [(0, 0), (N - 64, 8000), (8191, 12000)]:
+            ref = hotspot_window_block(T, P, i0, j0, 64, 64, n, coef)
+            got = out[i0:i0 + 64, j0:j0 + 64]
+            assert rel_err(got, ref) <= TOL, (g.astuple(), i0, j0, rel_err(got, ref))
+    finally:
+        oracle.set_threads(1)
 
 
 def test_host_entry_point(rg):

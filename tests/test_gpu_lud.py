@@ -156,3 +156,37 @@ def test_tc_full_size_backward_error(rg):
     Ad = torch.from_numpy(A[rows.cpu().numpy()].astype(np.float64)).to(p.device)
     err = float((Ad - L[rows] @ U).abs().max() / abs(A).max())
     assert err <= 1e-5, err
+
+
+def test_concurrent_calls_same_n_two_streams(rg):
+    # Two factorisations of the same size on two streams share one cached graph; each must
+    # factor its own matrix (the slot write is the graph's root node, updated per launch).
+    n = 2048
+    A1 = synth.lud_rodinia_matrix(n)
+    A2 = synth.lud_diag_dominant(n)
+    for panel in (16, 128):
+        r1 = _lu(rg, A1, panel).clone()
+        r2 = _lu(rg, A2, panel).clone()
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        for _ in range(3):
+            t1 = torch.from_numpy(A1).cuda()
+            t2 = torch.from_numpy(A2).cuda()
+            torch.cuda.synchronize()
+            rg.rodinia_lud(t1, panel, g=UNC, stream=s1)
+            rg.rodinia_lud(t2, panel, g=UNC, stream=s2)
+            torch.cuda.synchronize()
+            assert torch.equal(t1, r1) and torch.equal(t2, r2), panel
+
+
+def test_unaligned_matrix_view(rg):
+    # an offset view (not 16-byte aligned) is factored bit-identically to an aligned copy
+    n = 300
+    A = synth.lud_rodinia_matrix(n)
+    for panel in (16, 32, 128):
+        ref = _lu(rg, A, panel, (2, 2, 2, 2, 1, 1, 0) if panel != 128 else UNC)
+        buf = torch.empty(n * n + 1, device="cuda")
+        v = buf[1:].view(n, n)
+        v.copy_(torch.from_numpy(A))
+        rg.rodinia_lud(v, panel, g=(2, 2, 2, 2, 1, 1, 0) if panel != 128 else UNC)
+        torch.cuda.synchronize()
+        assert torch.equal(v, ref), panel

@@ -88,3 +88,21 @@ def test_tuner_returns_legal_bit_exact_choice(rg):
     assert any(r["status"] == 0 and r["median_ms"] > 0 for r in rows)
     wall = synth.pathfinder_wall(100, 100000)
     assert np.array_equal(_run(rg, wall, best), oracle.pathfinder(wall))
+
+
+def test_unaligned_views_bit_exact(rg):
+    # offset views of the wall and result (4 bytes off 16-byte alignment) take the scalar edge
+    # path of the warp-band kernel instead of faulting on 128-bit accesses
+    R, C = 60, 4096
+    wall = synth.pathfinder_wall(R, C, seed=8)
+    ref = oracle.pathfinder(wall)
+    wb = torch.zeros(R * C + 1, dtype=torch.int32, device="cuda")
+    w = wb[1:].view(R, C)
+    w.copy_(torch.from_numpy(wall))
+    ob = torch.zeros(C + 3, dtype=torch.int32, device="cuda")
+    for g in [(4, 1, 1, 1, 20, 1, 2), (2, 1, 1, 1, 12, 1, 2), (8, 1, 1, 1, 16, 1, 2)]:
+        out = rg.rodinia_pathfinder(w, g=g, out=ob[1:1 + C])
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy(), ref), g
+        aligned = rg.rodinia_pathfinder(torch.from_numpy(wall).cuda(), g=g)
+        assert np.array_equal(aligned.cpu().numpy(), ref), g

@@ -177,3 +177,72 @@ def test_srad_v1_smooths_speckle():
         return J.std() / J.mean()
     assert cv(out) < 0.8 * cv(img)
     assert out.min() >= img.min() - 1e-9 and out.max() <= img.max() + 1e-9  # maximum principle
+
+
+# ----------------------------------------------------------------------------- q0sqr per iteration
+def _row_mode(R, C, eps):
+    # J = 1 + eps*cos(pi*(i+1/2)/R): the slowest eigenmode of the clamped (Neumann) 5-point
+    # Laplacian along rows, constant along columns; eigenvalue -4 sin^2(pi/(2R))
+    i = np.arange(R, dtype=np.float64)[:, None]
+    return np.repeat(1.0 + eps * np.cos(np.pi * (i + 0.5) / R), C, axis=1)
+
+
+def test_q0sqr_is_reevaluated_every_iteration_closed_form():
+    # Rodinia srad_v2's host loop recomputes the ROI statistics at the top of EVERY iteration
+    # (DESIGN.md §3 S1/S2; SURVEY §8(c) srad definition "for it in 0..niter-1: ... s = sum_ROI J").
+    # On the row eigenmode with the ROI = whole grid, c saturates at 1 (qsqr ~ (eps*pi/R)^2 is
+    # far below q0sqr ~ eps^2/2), so J_t = 1 + eps g^t cos(.) with g = 1 - lambda sin^2(pi/2R):
+    # mean_t = 1 (sum of cos over the period is 0), var_t = eps^2 g^(2t) / 2, hence
+    #   q0sqr(t) = eps^2 g^(2t) / 2       (closed form, t = 0..niter-1).
+    # A "q0sqr computed once" oracle reports eps^2/2 at every t and fails from t = 1.
+    R, C, eps, lam, n = 64, 6, 0.25, 0.5, 6
+    J = _row_mode(R, C, eps)
+    out, q0 = oracle.srad(J, 0, R - 1, 0, C - 1, lam, n, return_q0=True)
+    g = 1.0 - lam * np.sin(np.pi / (2 * R)) ** 2
+    want = eps ** 2 * g ** (2 * np.arange(n)) / 2.0
+    np.testing.assert_allclose(q0, want, rtol=1e-10, atol=0)
+    assert q0[1] < q0[0] * (1 - 1e-4)  # the sequence really moves
+    np.testing.assert_allclose(out, 1.0 + (J - 1.0) * g ** n, rtol=0, atol=1e-13)
+
+
+def test_q0sqr_sequence_drives_later_iterations():
+    # composition with the independently pinned pieces: iteration t uses q0sqr of J_t (not of
+    # J_0).  Random data, ROI in a corner, so c is not saturated and q0 matters for J itself.
+    rng = np.random.default_rng(11)
+    J0 = np.exp(rng.random((24, 31)))
+    r1, r2, c1, c2, lam = 2, 9, 3, 12, 0.5
+    J = J0.copy()
+    seq = []
+    for _ in range(3):
+        q = oracle.srad_q0sqr(J, r1, r2, c1, c2)
+        seq.append(q)
+        J = oracle.srad_step(J, q, lam)
+    out, q0 = oracle.srad(J0, r1, r2, c1, c2, lam, 3, return_q0=True)
+    assert np.array_equal(q0, np.array(seq))
+    assert np.array_equal(out, J)
+    frozen = J0.copy()
+    for _ in range(3):  # the mutation: q0sqr of J_0 reused
+        frozen = oracle.srad_step(frozen, seq[0], lam)
+    assert np.abs(frozen - out).max() > 1e-6
+
+
+def test_srad_v1_extract_compress_scale_closed_form():
+    # Reading V1 (Rodinia srad_v1 `extract` J = exp(image/255), `compress` image = log(J)*255;
+    # the srad the paper evaluates).  Choose the image so that the extracted J is
+    # exactly the row eigenmode: image = 255*log(1 + eps cos(.)).  With the whole-image ROI, c
+    # saturates (as above) and J_t = 1 + eps g^t cos(.), so the compressed output is
+    #   image_t = 255 * log(1 + eps g^t cos(pi (i+1/2)/R)).
+    # Any other extract scale s makes J0 = (1 + eps cos)^(255/s), not an eigenmode; any other
+    # compress scale s' multiplies the output by s'/255: both fail this closed form.
+    R, C, eps, lam, n = 48, 5, 0.3, 0.5, 7
+    i = np.arange(R, dtype=np.float64)[:, None]
+    mode = np.repeat(np.cos(np.pi * (i + 0.5) / R), C, axis=1)
+    img = 255.0 * np.log(1.0 + eps * mode)
+    g = 1.0 - lam * np.sin(np.pi / (2 * R)) ** 2
+    want = 255.0 * np.log(1.0 + eps * g ** n * mode)
+    np.testing.assert_allclose(oracle.srad_v1(img, lam, n), want, rtol=0, atol=1e-10)
+    # negative controls: the same pin evaluated with scale 256 or natural-log units fails
+    for s in (256.0, 1.0):
+        J = np.exp(img / s)
+        bad = s * np.log(oracle.srad(J, 0, R - 1, 0, C - 1, lam, n))
+        assert np.abs(bad - want).max() > 1e-6
