@@ -310,6 +310,35 @@ rodinia_status rodinia_comm_init(rodinia_comm** out, int32_t nranks, int32_t ran
 rodinia_status rodinia_comm_init_local(rodinia_comm** out, int32_t nranks);
 rodinia_status rodinia_comm_destroy(rodinia_comm* comm);
 
+/* The schedule a rank follows (host only, no device needed):
+ *  row0, own          owned global rows [row0, row0 + own) (= rodinia_slab)
+ *  top, bot           halo rows stored above / below the owned rows
+ *  period             iterations between halo exchanges (the temporal depth D)
+ *  send_up, send_down rows sent per exchange to rank-1 (its first owned rows) / rank+1 (its last)
+ *  exchanges          exchanges in `iterations` (0 for one rank)
+ *  overlap            1 if the interior launch of a period overlaps its exchange (hotspot)
+ *  cone_*             srad: the ROI's dependency-cone window [cone_r0, cone_r1) x [cone_c0,
+ *                     cone_c1) every rank evolves to obtain q0sqr(t) (reading S10); 0 for hotspot
+ * hotspot: D = steps per launch of the granularity, halos D / D, sends D / D.
+ * srad: D = granularity temporal (a NULL/zero granularity: min(8, rows per slab / 2)), halos D
+ * above / 2D below (one iteration reads rows i-1..i+2), sends 2D up / D down.
+ * r1..c2: the srad ROI (ignored for hotspot).  Errors: RODINIA_E_INVALID (arguments, other
+ * kernels: pathfinder and lud are replicas only), RODINIA_E_ILLEGAL_FACTOR (slab thinner than the
+ * halo), granularity errors as for the single-GPU call. */
+typedef struct {
+    int64_t row0, own;
+    int32_t top, bot;
+    int32_t period;
+    int32_t send_up, send_down;
+    int32_t exchanges;
+    int32_t overlap;
+    int32_t reserved;
+    int64_t cone_r0, cone_r1, cone_c0, cone_c1;
+} rodinia_dist_plan;
+rodinia_status rodinia_dist_schedule(rodinia_kernel k, int64_t global_rows, int64_t cols, int32_t nranks,
+                                 int32_t rank, int32_t iterations, int64_t r1, int64_t r2, int64_t c1,
+                                 int64_t c2, const rodinia_granularity* g, rodinia_dist_plan* out);
+
 /* NCCL communicator: temp_local/power_local/out_local hold this rank's slab (rodinia_slab
  * rows x cols).  Local communicator: the pointers are arrays of `nranks` slab pointers
  * (const float* const*), passed as the same arguments.  Bitwise equal to rodinia_hotspot
@@ -319,6 +348,10 @@ rodinia_status rodinia_hotspot_dist(rodinia_comm* comm, const void* temp_local,
                                     int64_t global_rows, int64_t cols, int32_t iterations,
                                     const rodinia_hotspot_coeffs* coeffs,
                                     const rodinia_granularity* g, void* stream);
+/* srad on row slabs: J_local is this rank's slab (LOCAL: array of slab pointers), updated in
+ * place; g->temporal (>= 1) is the exchange period D (each launch is still one iteration), a
+ * NULL/zero granularity picks the tuned kernel and D = min(8, rows per slab / 2).  Bitwise equal
+ * to rodinia_srad on the whole grid with the same kernel granularity. */
 rodinia_status rodinia_srad_dist(rodinia_comm* comm, void* J_local, int64_t global_rows,
                                  int64_t cols, int64_t r1, int64_t r2, int64_t c1, int64_t c2,
                                  float lambda, int32_t niter, const rodinia_granularity* g,

@@ -1,5 +1,6 @@
 // dist.cu -- multi-GPU row-slab decomposition for the stencils (hotspot, srad), one process
-// per GPU, NCCL point-to-point halo exchange over NVLink / NVSwitch.
+// per GPU, NCCL point-to-point halo exchange over NVLink / NVSwitch (SURVEY §8(e)
+// and §8(a) S13).
 //
 // Rank r owns global rows [floor(r*R/P), floor((r+1)*R/P)).  Its local buffer is
 //   [top halo][own rows][bottom halo]
@@ -7,17 +8,24 @@
 // single-GPU path runs on a slab: rows next to a non-global buffer edge go stale by one row
 // (hotspot; srad: one row at the top, two at the bottom) per step, which the halo depth absorbs.
 //  * hotspot: halo D = steps fused per launch (temporal); every D steps each rank sends its
-//    first D own rows up and its last D own rows down (ncclSend/ncclRecv in one group on the
-//    compute stream).  Power halos are exchanged once.
-//  * srad: one iteration reads rows i-1..i+2, so halos are D above and 2D below.  The global
-//    ROI statistics q0sqr(t) are computed without any per-iteration collective: every rank
-//    gathers the ROI's dependency cone of J0 once (rows [r1-n, r2+2n+2] x cols likewise,
+//    first D own rows up and its last D own rows down (ncclSend/ncclRecv in one group).  The
+//    exchange overlaps the interior launch: the owned rows alone determine output rows
+//    [D, own-D) after D steps, so the interior runs on the compute stream while a side stream
+//    exchanges the halos and then computes the two boundary strips (D halo rows + 2D owned rows
+//    each) into strip buffers; the compute stream copies their D valid rows in after the
+//    interior.  Power halos are exchanged once per call.
+//  * srad: one iteration reads rows i-1..i+2, so halos are D above and 2D below, exchanged
+//    every D iterations (D = the granularity's temporal depth; default min(8, own/2)).  The
+//    global ROI statistics q0sqr(t) are computed without any per-iteration collective: every
+//    rank gathers the ROI's dependency cone of J0 once (rows [r1-n, r2+2n+2] x cols likewise,
 //    ncclBroadcast from the owners) and evolves just that window with the same kernels; ROI
 //    values on the window are bit-identical to the full grid (reading S10), hence so is q0sqr(t).
-// Results are bitwise identical to the single-GPU call with the same granularity.
+// Results are bitwise identical to the single-GPU call with the same granularity.  The slab
+// buffers, strip buffers, srad engines and the side stream live in the communicator and are
+// reused by later calls of the same shape (no per-call allocation after the first).
 //
 // A second communicator kind, LOCAL, keeps all P slabs on the current device and moves halos
-// with cudaMemcpyAsync; it exercises the identical slab/halo logic on one GPU (tests).
+// with cudaMemcpyAsync; it runs the identical slab/halo/overlap logic on one GPU (tests).
 //
 // NCCL is not linked: libnccl.so.2 is dlopen'ed at run time (the copy torch already mapped,
 // or $RODINIA_NCCL_LIB), so the library loads on hosts without NCCL.
@@ -27,16 +35,50 @@
 #include <string.h>
 
 #include <algorithm>
+#include <cmath>
 #include <mutex>
 #include <vector>
 
 #include "rg_internal.h"
 #include "workloads.h"
 
+namespace rg {
+struct Slab {
+    int rank;       // global slab index
+    int64_t row0;   // first owned global row
+    int own;        // owned rows
+    int top, bot;   // halo rows above / below
+    float* buf[2];  // local buffers (top + own + bot rows)
+    float* aux;     // hotspot: pre-scaled power kP; unused for srad
+    float* scr;     // hotspot: ping-pong scratch for multi-launch periods
+    float* strip[2];     // hotspot overlap: boundary-strip outputs (top, bottom), 3D rows each
+    float* strip_scr;    // ... and their ping-pong scratch
+    int rows() const { return top + own + bot; }
+};
+namespace srad { struct Engine; }
+}  // namespace rg
+
 struct rodinia_comm {
     int kind;  // 0 = NCCL (one slab per process), 1 = LOCAL (all slabs in this process)
     int nranks, rank;
     ncclComm_t nccl;
+    std::mutex mu;
+    int dev = -1;
+    cudaStream_t side = nullptr;          // exchange + boundary strips (hotspot overlap)
+    cudaEvent_t ev_ready = nullptr, ev_strips = nullptr;
+    cudaEvent_t ev_done = nullptr;        // end of the previous call (orders calls on any stream)
+    bool done_recorded = false;
+    // persistent buffers of the last shape (hotspot and srad separately)
+    struct HsCache { int64_t R = 0, C = 0; int D = 0; std::vector<rg::Slab> sl; } hs;
+    struct SrCache {
+        int64_t R = 0, C = 0; int D = 0, niter_cap = 0, WR = 0, WC = 0;
+        rodinia_granularity g{};
+        std::vector<rg::Slab> sl;
+        std::vector<rg::srad::Engine> eng;
+        rg::srad::Engine we;
+        float* W = nullptr;
+        bool have_we = false;
+    } sr;
 };
 
 namespace rg {
@@ -97,23 +139,49 @@ static rodinia_status nccl_api(NcclApi** out) {
         if (_r != ncclSuccess) return set_error(RODINIA_E_NCCL, "%s: %s", #x, (api)->GetErrorString(_r)); \
     } while (0)
 
-// ------------------------------------------------------------------ slabs
+// ------------------------------------------------------------------ slabs and plans (host only)
 static void slab_of(int64_t R, int P, int r, int64_t* row0, int64_t* n) {
     const int64_t a = (int64_t)r * R / P, b = (int64_t)(r + 1) * R / P;
     *row0 = a;
     *n = b - a;
 }
 
-struct Slab {
-    int rank;       // global slab index
-    int64_t row0;   // first owned global row
-    int own;        // owned rows
-    int top, bot;   // halo rows above / below
-    float* buf[2];  // local buffers (top + own + bot rows)
-    float* aux;     // hotspot: power; unused for srad
-    float* scr;     // hotspot: ping-pong scratch for multi-launch periods
-    int rows() const { return top + own + bot; }
-};
+// The schedule of one rank (rodinia_dist_plan): halo depths, exchange period and sizes.
+//  hotspot: D = steps per launch of the granularity; halos D / D; sends D / D rows.
+//  srad:    D = exchange period; halos D above / 2D below; sends 2D rows up, D down; cone window.
+static rodinia_status plan_of(rodinia_kernel k, int64_t R, int64_t C, int P, int r, int iters, int64_t r1,
+                              int64_t r2, int64_t c1, int64_t c2, int D, rodinia_dist_plan* o) {
+    memset(o, 0, sizeof *o);
+    slab_of(R, P, r, &o->row0, &o->own);
+    const int up = k == RODINIA_SRAD ? 2 * D : D;  // rows a slab sends to the rank above
+    const int down = D;                           // rows a slab sends to the rank below
+    o->period = D;
+    o->top = r > 0 ? down : 0;
+    o->bot = r + 1 < P ? up : 0;
+    o->send_up = r > 0 ? up : 0;
+    o->send_down = r + 1 < P ? down : 0;
+    o->exchanges = P > 1 ? (iters + D - 1) / D : 0;
+    int64_t own_min = R / P;  // smallest slab
+    if (P > 1 && own_min < std::max(up, down))
+        return set_error(RODINIA_E_ILLEGAL_FACTOR,
+                         "dist: slabs of %lld rows are thinner than the halo depth %d; use fewer ranks or a "
+                         "smaller temporal depth", (long long)own_min, std::max(up, down));
+    // hotspot overlap: the owned rows determine output rows [D, own - D) by themselves
+    o->overlap = (k == RODINIA_HOTSPOT && P > 1 && o->own > 2 * D) ? 1 : 0;
+    if (k == RODINIA_SRAD) {
+        o->cone_r0 = std::max<int64_t>(0, r1 - iters);
+        o->cone_r1 = std::min<int64_t>(R, r2 + 2 * (int64_t)iters + 3);
+        o->cone_c0 = std::max<int64_t>(0, c1 - iters);
+        o->cone_c1 = std::min<int64_t>(C, c2 + 2 * (int64_t)iters + 3);
+    }
+    return RODINIA_OK;
+}
+
+static int srad_auto_depth(int64_t R, int P) {
+    if (P == 1) return 1;
+    const int64_t own_min = R / P;
+    return (int)std::max<int64_t>(1, std::min<int64_t>(8, own_min / 2));
+}
 
 // Halo exchange of buffer `which` of every local slab: every slab sends its first `up` own
 // rows to the slab above (its bottom halo, depth up) and its last `down` own rows to the slab
@@ -157,7 +225,24 @@ static rodinia_status exchange(rodinia_comm* c, std::vector<Slab>& sl, int which
     return RODINIA_OK;
 }
 
-static rodinia_status make_slabs(rodinia_comm* c, int64_t R, int up, int down, std::vector<Slab>* out) {
+static void free_slab(Slab& x) {
+    for (float* p : {x.buf[0], x.buf[1], x.aux, x.scr, x.strip[0], x.strip[1], x.strip_scr})
+        if (p) cudaFree(p);
+    memset(&x, 0, sizeof x);
+}
+
+static rodinia_status dev_alloc(float** p, size_t floats) {
+    if (cudaMalloc((void**)p, std::max<size_t>(floats, 1) * sizeof(float)) != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return set_error(RODINIA_E_NOMEM, "dist: slab allocation of %zu floats failed", floats);
+    }
+    return RODINIA_OK;
+}
+
+// The slabs this process holds (NCCL: its own; LOCAL: all), with halo depths from the plan.
+static rodinia_status make_slabs(rodinia_comm* c, rodinia_kernel k, int64_t R, int64_t C, int iters, int D,
+                                 std::vector<Slab>* out) {
     const int P = c->nranks;
     std::vector<int> ranks;
     if (c->kind == 1)
@@ -165,30 +250,31 @@ static rodinia_status make_slabs(rodinia_comm* c, int64_t R, int up, int down, s
     else
         ranks.push_back(c->rank);
     for (int r : ranks) {
+        rodinia_dist_plan pl;
+        RG_TRY(plan_of(k, R, C, P, r, iters, 0, 0, 0, 0, D, &pl));
         Slab x;
         memset(&x, 0, sizeof x);
         x.rank = r;
-        int64_t n;
-        slab_of(R, P, r, &x.row0, &n);
-        x.own = (int)n;
-        x.top = r > 0 ? down : 0;
-        x.bot = r + 1 < P ? up : 0;
-        if (P > 1 && x.own < std::max(up, down))
-            return set_error(RODINIA_E_ILLEGAL_FACTOR,
-                             "dist: slab %d has %d rows, fewer than the halo depth %d; use fewer ranks or a "
-                             "smaller temporal depth", r, x.own, std::max(up, down));
+        x.row0 = pl.row0;
+        x.own = (int)pl.own;
+        x.top = pl.top;
+        x.bot = pl.bot;
         out->push_back(x);
     }
     return RODINIA_OK;
 }
 
-static void free_slabs(std::vector<Slab>& sl, cudaStream_t s) {
-    for (auto& x : sl) {
-        scratch_free(x.buf[0], s);
-        scratch_free(x.buf[1], s);
-        scratch_free(x.aux, s);
-        scratch_free(x.scr, s);
-    }
+static rodinia_status comm_setup(rodinia_comm* c) {
+    int dev = 0;
+    RG_CUDA(cudaGetDevice(&dev));
+    if (c->side && c->dev == dev) return RODINIA_OK;
+    RG_CUDA(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+    RG_CUDA(cudaEventCreateWithFlags(&c->ev_ready, cudaEventDisableTiming));
+    RG_CUDA(cudaEventCreateWithFlags(&c->ev_strips, cudaEventDisableTiming));
+    RG_CUDA(cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming));
+    c->dev = dev;
+    c->done_recorded = false;
+    return RODINIA_OK;
 }
 
 // pointer of local slab i among the caller's arguments (NCCL: the pointer itself; LOCAL: array)
@@ -205,6 +291,61 @@ extern "C" rodinia_status rodinia_slab(int64_t R, int32_t P, int32_t r, int64_t*
     if (R < 1 || P < 1 || r < 0 || r >= P || !row0 || !nrows) return set_error(RODINIA_E_INVALID, "slab: bad arguments");
     slab_of(R, P, r, row0, nrows);
     return RODINIA_OK;
+}
+
+static rodinia_status resolve_hotspot(int64_t R, int64_t C, int iters, int P, const rodinia_granularity* g,
+                                      rodinia_granularity* gg, const hotspot::DirectVariant** dv,
+                                      const hotspot::StreamVariant** sv) {
+    int64_t row0, own0;
+    slab_of(R, P, 0, &row0, &own0);
+    if (!gran_is_zero(g)) *gg = *g;
+    else {
+        rodinia_problem pb{own0, C, iters, P};
+        if (!tune_cache_lookup(RODINIA_HOTSPOT, pb, gg)) *gg = default_gran(RODINIA_HOTSPOT, pb);
+    }
+    // the largest buffer a launch sees: the biggest slab with both halos
+    const int h = (gg->flags & RODINIA_STREAM) ? std::max(1, gg->temporal) : 1;
+    return hotspot::check(*gg, (R + P - 1) / P + 2 * h, C, dv, sv);
+}
+
+static rodinia_status resolve_srad(int64_t R, int64_t C, int niter, int P, const rodinia_granularity* g,
+                                   rodinia_granularity* gg, int* D) {
+    int64_t row0, own0;
+    slab_of(R, P, 0, &row0, &own0);
+    if (!gran_is_zero(g)) {
+        *gg = *g;
+        *D = std::max(1, g->temporal);  // exchange period / halo depth
+    } else {
+        rodinia_problem pb{own0, C, niter, P};
+        if (!tune_cache_lookup(RODINIA_SRAD, pb, gg)) *gg = default_gran(RODINIA_SRAD, pb);
+        *D = srad_auto_depth(R, P);
+    }
+    gg->temporal = 1;  // every srad launch is one iteration; D only sets the exchange period
+    return RODINIA_OK;
+}
+
+extern "C" rodinia_status rodinia_dist_schedule(rodinia_kernel k, int64_t R, int64_t C, int32_t P, int32_t r,
+                                            int32_t iters, int64_t r1, int64_t r2, int64_t c1, int64_t c2,
+                                            const rodinia_granularity* g, rodinia_dist_plan* out) {
+    if (!out || R < 1 || C < 1 || P < 1 || r < 0 || r >= P || iters < 0 || R < P)
+        return set_error(RODINIA_E_INVALID, "dist_schedule: bad arguments");
+    if (k == RODINIA_HOTSPOT) {
+        rodinia_granularity gg;
+        const hotspot::DirectVariant* dv;
+        const hotspot::StreamVariant* sv;
+        RG_TRY(resolve_hotspot(R, C, iters, P, g, &gg, &dv, &sv));
+        return plan_of(k, R, C, P, r, iters, 0, 0, 0, 0, hotspot::temporal_of(sv), out);
+    }
+    if (k == RODINIA_SRAD) {
+        if (r1 < 0 || c1 < 0 || r2 < r1 || c2 < c1 || r2 >= R || c2 >= C)
+            return set_error(RODINIA_E_INVALID, "dist_schedule: ROI outside the grid");
+        rodinia_granularity gg;
+        int D;
+        RG_TRY(resolve_srad(R, C, iters, P, g, &gg, &D));
+        return plan_of(k, R, C, P, r, iters, r1, r2, c1, c2, D, out);
+    }
+    return set_error(RODINIA_E_INVALID, "dist_schedule: only hotspot and srad are sharded (pathfinder and lud run "
+                                        "as replicas, DESIGN.md §6)");
 }
 
 extern "C" rodinia_status rodinia_comm_unique_id(uint8_t id[128]) {
@@ -250,17 +391,85 @@ extern "C" rodinia_status rodinia_comm_init_local(rodinia_comm** out, int32_t nr
     return RODINIA_OK;
 }
 
+static void release_hs(rodinia_comm* c) {
+    for (auto& x : c->hs.sl) free_slab(x);
+    c->hs.sl.clear();
+    c->hs.R = c->hs.C = 0;
+}
+
+static void release_sr(rodinia_comm* c) {
+    for (auto& x : c->sr.sl) {
+        x.buf[1] = nullptr;  // the engine's ping-pong buffer (freed with the engine)
+        free_slab(x);
+    }
+    for (auto& e : c->sr.eng) srad::engine_free(&e, nullptr);
+    if (c->sr.have_we) srad::engine_free(&c->sr.we, nullptr);
+    if (c->sr.W) cudaFree(c->sr.W);
+    c->sr.sl.clear();
+    c->sr.eng.clear();
+    c->sr.W = nullptr;
+    c->sr.have_we = false;
+    c->sr.R = c->sr.C = 0;
+}
+
 extern "C" rodinia_status rodinia_comm_destroy(rodinia_comm* c) {
     if (!c) return set_error(RODINIA_E_INVALID, "comm_destroy: null");
-    if (c->kind == 0 && c->nccl) {
-        NcclApi* api;
-        if (nccl_api(&api) == RODINIA_OK) api->CommDestroy(c->nccl);
+    {
+        std::lock_guard<std::mutex> lk(c->mu);
+        if (c->side) {
+            cudaDeviceSynchronize();  // buffers may still be in use by enqueued work
+            release_hs(c);
+            release_sr(c);
+            cudaStreamDestroy(c->side);
+            cudaEventDestroy(c->ev_ready);
+            cudaEventDestroy(c->ev_strips);
+            cudaEventDestroy(c->ev_done);
+            cudaGetLastError();  // teardown errors are not reported to later calls
+        }
+        if (c->kind == 0 && c->nccl) {
+            NcclApi* api;
+            if (nccl_api(&api) == RODINIA_OK) api->CommDestroy(c->nccl);
+        }
     }
     delete c;
     return RODINIA_OK;
 }
 
 // ===================================================================== exported: hotspot_dist
+// One full period with overlap: side stream = exchange + boundary strips into
+// strip buffers, compute stream = interior launch on the owned rows, then the strips' valid
+// rows are copied into the output buffer.
+static rodinia_status hs_period_overlap(rodinia_comm* c, std::vector<Slab>& sl, int cur, int C, int D,
+                                        const HsCoef& cf, const rodinia_granularity& gg,
+                                        const hotspot::DirectVariant* dv, const hotspot::StreamVariant* sv,
+                                        cudaStream_t s) {
+    const size_t rowb = (size_t)C * sizeof(float);
+    RG_CUDA(cudaEventRecord(c->ev_ready, s));
+    RG_CUDA(cudaStreamWaitEvent(c->side, c->ev_ready, 0));
+    RG_TRY(exchange(c, sl, cur, C, D, D, false, c->side));
+    for (auto& x : sl) {
+        // top strip: buffer rows [0, top + 2D) -> outputs [top, top + D)
+        const int tr = x.top + 2 * D;
+        RG_TRY(hotspot::run(x.buf[cur], x.aux, x.strip[0], x.strip_scr, tr, C, D, cf, gg, dv, sv, c->side));
+        // bottom strip: buffer rows [top + own - 2D, rows) -> outputs [D, 2D) of the strip
+        const int b0 = x.top + x.own - 2 * D, br = 2 * D + x.bot;
+        RG_TRY(hotspot::run(x.buf[cur] + (size_t)b0 * C, x.aux + (size_t)b0 * C, x.strip[1], x.strip_scr, br, C, D,
+                            cf, gg, dv, sv, c->side));
+    }
+    RG_CUDA(cudaEventRecord(c->ev_strips, c->side));
+    for (auto& x : sl)  // interior: the owned rows alone, outputs [D, own - D) valid
+        RG_TRY(hotspot::run(x.buf[cur] + (size_t)x.top * C, x.aux + (size_t)x.top * C,
+                            x.buf[1 - cur] + (size_t)x.top * C, x.scr, x.own, C, D, cf, gg, dv, sv, s));
+    RG_CUDA(cudaStreamWaitEvent(s, c->ev_strips, 0));
+    for (auto& x : sl) {
+        RG_CUDA(cudaMemcpyAsync(x.buf[1 - cur] + (size_t)x.top * C, x.strip[0] + (size_t)x.top * C, D * rowb,
+                                cudaMemcpyDeviceToDevice, s));
+        RG_CUDA(cudaMemcpyAsync(x.buf[1 - cur] + (size_t)(x.top + x.own - D) * C, x.strip[1] + (size_t)D * C,
+                                D * rowb, cudaMemcpyDeviceToDevice, s));
+    }
+    return RODINIA_OK;
+}
+
 extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp_local, const void* power_local,
                                                void* out_local, int64_t R, int64_t C, int32_t iters,
                                                const rodinia_hotspot_coeffs* coeffs, const rodinia_granularity* g,
@@ -273,51 +482,66 @@ extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp
             if (!arg_ptr(c, temp_local, i) || !arg_ptr(c, power_local, i) || !((float* const*)out_local)[i])
                 return set_error(RODINIA_E_INVALID, "hotspot_dist: null slab pointer");
     rodinia_granularity gg;
-    int64_t row0, own0;
-    slab_of(R, c->nranks, 0, &row0, &own0);
-    if (!gran_is_zero(g)) gg = *g;
-    else {
-        rodinia_problem pb{own0, C, iters, c->nranks};
-        if (!tune_cache_lookup(RODINIA_HOTSPOT, pb, &gg)) gg = default_gran(RODINIA_HOTSPOT, pb);
-    }
     const hotspot::DirectVariant* dv;
     const hotspot::StreamVariant* sv;
-    RG_TRY(hotspot::check(gg, own0 + 2 * 64, C, &dv, &sv));
+    RG_TRY(resolve_hotspot(R, C, iters, c->nranks, g, &gg, &dv, &sv));
     const int D = hotspot::temporal_of(sv);
     rodinia_hotspot_coeffs cc;
     if (coeffs) cc = *coeffs;
     else rodinia_hotspot_coeffs_rodinia(R, C, 0.016, 0.016, &cc);
     const HsCoef cf = hs_derive(cc.k, cc.rx, cc.ry, cc.rz);  // state form (hs_cell.cuh)
-    std::vector<Slab> sl;
-    RG_TRY(make_slabs(c, R, D, D, &sl));
+    std::vector<Slab> want;
+    RG_TRY(make_slabs(c, RODINIA_HOTSPOT, R, C, iters, D, &want));
     DeviceInfo di;
     RG_TRY(device_info(&di));
+    std::lock_guard<std::mutex> lk(c->mu);
+    RG_TRY(comm_setup(c));
     cudaStream_t s = (cudaStream_t)stream;
-    const size_t rowb = (size_t)C * sizeof(float);
-    rodinia_status st = RODINIA_OK;
-    for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
-        Slab& x = sl[i];
-        const size_t bytes = (size_t)x.rows() * rowb;
-        st = scratch_alloc((void**)&x.buf[0], bytes, s);
-        if (st == RODINIA_OK) st = scratch_alloc((void**)&x.buf[1], bytes, s);
-        if (st == RODINIA_OK) st = scratch_alloc((void**)&x.aux, bytes, s);
-        if (st == RODINIA_OK) st = scratch_alloc((void**)&x.scr, bytes, s);
-        if (st == RODINIA_OK) {
-            cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, arg_ptr(c, temp_local, i), x.own * rowb, cudaMemcpyDeviceToDevice, s);
-            cudaMemcpyAsync(x.aux + (size_t)x.top * C, arg_ptr(c, power_local, i), x.own * rowb, cudaMemcpyDeviceToDevice, s);
-            // T -> u = T - amb and P -> kP = k*P on the owned rows (halos arrive converted)
-            hotspot::convert(x.buf[0] + (size_t)x.top * C, x.buf[0] + (size_t)x.top * C, (int64_t)x.own * C, 0, cc.amb, s);
-            hotspot::convert(x.aux + (size_t)x.top * C, x.aux + (size_t)x.top * C, (int64_t)x.own * C, 1, cc.k, s);
+    // the communicator's buffers are reused: order this call after the previous one
+    if (c->done_recorded) RG_CUDA(cudaStreamWaitEvent(s, c->ev_done, 0));
+    // persistent slab buffers (reallocated only when the shape or halo depth changes)
+    auto& hc = c->hs;
+    if (hc.R != R || hc.C != C || hc.D != D || hc.sl.size() != want.size()) {
+        RG_CUDA(cudaStreamSynchronize(s));
+        release_hs(c);
+        for (auto& x : want) {
+            const size_t n = (size_t)x.rows() * C, ns = (size_t)(x.top + 2 * D + std::max(x.bot, D)) * C;
+            RG_TRY(dev_alloc(&x.buf[0], n));
+            RG_TRY(dev_alloc(&x.buf[1], n));
+            RG_TRY(dev_alloc(&x.aux, n));
+            RG_TRY(dev_alloc(&x.scr, n));
+            RG_TRY(dev_alloc(&x.strip[0], ns));
+            RG_TRY(dev_alloc(&x.strip[1], ns));
+            RG_TRY(dev_alloc(&x.strip_scr, ns));
+            hc.sl.push_back(x);
         }
+        hc.R = R;
+        hc.C = C;
+        hc.D = D;
     }
-    if (st == RODINIA_OK && c->nranks > 1) st = exchange(c, sl, 0, (int)C, D, D, true, s);
+    std::vector<Slab>& sl = hc.sl;
+    const size_t rowb = (size_t)C * sizeof(float);
+    for (size_t i = 0; i < sl.size(); ++i) {
+        Slab& x = sl[i];
+        // T -> u = T - amb and P -> kP = k*P straight into the owned rows (halos arrive converted)
+        hotspot::convert(arg_ptr(c, temp_local, i), x.buf[0] + (size_t)x.top * C, (int64_t)x.own * C, 0, cc.amb, s);
+        hotspot::convert(arg_ptr(c, power_local, i), x.aux + (size_t)x.top * C, (int64_t)x.own * C, 1, cc.k, s);
+    }
+    rodinia_status st = RODINIA_OK;
+    if (c->nranks > 1) st = exchange(c, sl, 0, (int)C, D, D, true, s);
+    bool overlap = c->nranks > 1;
+    for (auto& x : sl) overlap = overlap && x.own > 2 * D;
     int cur = 0;
     for (int done = 0; st == RODINIA_OK && done < iters;) {
         const int steps = std::min(D, iters - done);
-        if (c->nranks > 1) st = exchange(c, sl, cur, (int)C, D, D, false, s);
-        for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
-            Slab& x = sl[i];
-            st = hotspot::run(x.buf[cur], x.aux, x.buf[1 - cur], x.scr, x.rows(), (int)C, steps, cf, gg, dv, sv, s);
+        if (overlap && steps == D && hotspot::num_launches(D, sv) == 1) {
+            st = hs_period_overlap(c, sl, cur, (int)C, D, cf, gg, dv, sv, s);
+        } else {
+            if (c->nranks > 1) st = exchange(c, sl, cur, (int)C, D, D, false, s);
+            for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
+                Slab& x = sl[i];
+                st = hotspot::run(x.buf[cur], x.aux, x.buf[1 - cur], x.scr, x.rows(), (int)C, steps, cf, gg, dv, sv, s);
+            }
         }
         cur = 1 - cur;
         done += steps;
@@ -326,11 +550,13 @@ extern "C" rodinia_status rodinia_hotspot_dist(rodinia_comm* c, const void* temp
         Slab& x = sl[i];
         float* dst = c->kind == 1 ? ((float* const*)out_local)[i] : (float*)out_local;
         hotspot::convert(x.buf[cur] + (size_t)x.top * C, dst, (int64_t)x.own * C, 2, cc.amb, s);  // u -> T
-        const cudaError_t ce = cudaGetLastError();
-        if (ce != cudaSuccess) st = cuda_error(ce, "hotspot_dist copy-out", __FILE__, __LINE__);
     }
-    if (st == RODINIA_OK && cudaGetLastError() != cudaSuccess) st = set_error(RODINIA_E_CUDA, "hotspot_dist: launch failed");
-    free_slabs(sl, s);
+    (void)rowb;
+    if (cudaEventRecord(c->ev_done, s) == cudaSuccess) c->done_recorded = true;
+    if (st == RODINIA_OK) {
+        const cudaError_t ce = cudaGetLastError();
+        if (ce != cudaSuccess) st = cuda_error(ce, "hotspot_dist", __FILE__, __LINE__);
+    }
     return st;
 }
 
@@ -340,6 +566,7 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
                                             const rodinia_granularity* g, void* stream) {
     if (!c || !J_local) return set_error(RODINIA_E_INVALID, "srad_dist: null argument");
     if (R < 1 || C < 1 || niter < 0 || R < c->nranks) return set_error(RODINIA_E_INVALID, "srad_dist: bad sizes");
+    if (R > (1ll << 31) - 1 || C > (1ll << 31) - 1) return set_error(RODINIA_E_INVALID, "srad_dist: grid too large");
     if (r1 < 0 || c1 < 0 || r2 < r1 || c2 < c1 || r2 >= R || c2 >= C)
         return set_error(RODINIA_E_INVALID, "srad_dist: ROI outside the grid");
     if (!std::isfinite(lambda)) return set_error(RODINIA_E_INVALID, "srad_dist: lambda not finite");
@@ -347,82 +574,96 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
         for (int i = 0; i < c->nranks; ++i)
             if (!((float* const*)J_local)[i]) return set_error(RODINIA_E_INVALID, "srad_dist: null slab pointer");
     rodinia_granularity gg;
-    int64_t row0, own0;
-    slab_of(R, c->nranks, 0, &row0, &own0);
-    if (!gran_is_zero(g)) gg = *g;
-    else {
-        rodinia_problem pb{own0, C, niter, c->nranks};
-        if (!tune_cache_lookup(RODINIA_SRAD, pb, &gg)) gg = default_gran(RODINIA_SRAD, pb);
-    }
+    int D;
+    RG_TRY(resolve_srad(R, C, niter, c->nranks, g, &gg, &D));
     srad::Plan p;
     RG_TRY(srad::plan(gg, &p));
-    if (p.v && p.smem > 48 * 1024)
-        RG_CUDA(cudaFuncSetAttribute((const void*)p.v->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem));
-    const int D = 1;  // exchange every iteration (halo 1 row above, 2 below)
-    std::vector<Slab> sl;
-    RG_TRY(make_slabs(c, R, 2 * D, D, &sl));
+    std::vector<Slab> want;
+    RG_TRY(make_slabs(c, RODINIA_SRAD, R, C, niter, D, &want));
     DeviceInfo di;
     RG_TRY(device_info(&di));
     RG_TRY(srad::take_sticky());
     if (niter == 0) return RODINIA_OK;
+    if (p.v && p.smem > 48 * 1024)
+        RG_CUDA(cudaFuncSetAttribute((const void*)p.v->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem));
+    std::lock_guard<std::mutex> lk(c->mu);
+    RG_TRY(comm_setup(c));
     cudaStream_t s = (cudaStream_t)stream;
     const size_t rowb = (size_t)C * sizeof(float);
+    if (c->done_recorded) RG_CUDA(cudaStreamWaitEvent(s, c->ev_done, 0));  // buffers are reused
+
+    // ---- the ROI's dependency-cone window (plan_of: rows [r1-n, r2+2n+3) x cols likewise)
+    rodinia_dist_plan pl0;
+    RG_TRY(plan_of(RODINIA_SRAD, R, C, c->nranks, 0, niter, r1, r2, c1, c2, D, &pl0));
+    const int64_t wr0 = pl0.cone_r0, wr1 = pl0.cone_r1, wc0 = pl0.cone_c0, wc1 = pl0.cone_c1;
+    const int WR = (int)(wr1 - wr0), WC = (int)(wc1 - wc0);
+
+    // ---- persistent slabs, engines and window (reallocated when the shape / plan changes)
+    auto& sc = c->sr;
+    const bool same = sc.R == R && sc.C == C && sc.D == D && sc.niter_cap >= niter && sc.WR == WR && sc.WC == WC &&
+                      !memcmp(&sc.g, &gg, sizeof gg) && sc.sl.size() == want.size();
+    if (!same) {
+        RG_CUDA(cudaStreamSynchronize(s));
+        release_sr(c);
+        for (auto& x : want) {
+            RG_TRY(dev_alloc(&x.buf[0], (size_t)x.rows() * C));
+            sc.sl.push_back(x);
+        }
+        sc.eng.resize(want.size());
+        for (size_t i = 0; i < want.size(); ++i) {
+            RG_TRY(srad::engine_alloc(&sc.eng[i], p, sc.sl[i].rows(), (int)C, niter, s));
+            sc.sl[i].buf[1] = sc.eng[i].jb;
+        }
+        RG_TRY(dev_alloc(&sc.W, (size_t)WR * WC));
+        RG_TRY(srad::engine_alloc(&sc.we, p, WR, WC, niter, s));
+        sc.have_we = true;
+        sc.R = R; sc.C = C; sc.D = D; sc.niter_cap = niter; sc.WR = WR; sc.WC = WC; sc.g = gg;
+    }
+    std::vector<Slab>& sl = sc.sl;
     rodinia_status st = RODINIA_OK;
 
     // ---- q0sqr(t) from the ROI's dependency cone (no per-iteration collective)
-    const int64_t wr0 = std::max<int64_t>(0, r1 - niter), wr1 = std::min<int64_t>(R, r2 + 2 * (int64_t)niter + 3);
-    const int64_t wc0 = std::max<int64_t>(0, c1 - niter), wc1 = std::min<int64_t>(C, c2 + 2 * (int64_t)niter + 3);
-    const int WR = (int)(wr1 - wr0), WC = (int)(wc1 - wc0);
-    float* W = nullptr;
-    srad::Engine we;
-    RG_TRY(scratch_alloc((void**)&W, (size_t)WR * WC * sizeof(float), s));
-    st = srad::engine_alloc(&we, p, WR, WC, niter, s);
-    if (st == RODINIA_OK) {
-        NcclApi* api = nullptr;
-        if (c->kind == 0 && c->nranks > 1) st = nccl_api(&api);
-        if (st == RODINIA_OK && api) {
-            ncclResult_t r = api->GroupStart();
-            for (int q = 0; q < c->nranks && r == ncclSuccess; ++q) {
-                int64_t q0, qn;
-                slab_of(R, c->nranks, q, &q0, &qn);
-                const int64_t a = std::max(q0, wr0), b = std::min(q0 + qn, wr1);
-                if (a >= b) continue;
-                float* part = W + (size_t)(a - wr0) * WC;
-                if (q == c->rank)  // owner packs its rows of the window
-                    cudaMemcpy2DAsync(part, WC * sizeof(float), (const float*)J_local + (size_t)(a - q0) * C + wc0,
-                                      rowb, WC * sizeof(float), (size_t)(b - a), cudaMemcpyDeviceToDevice, s);
-                r = api->Bcast(part, part, (size_t)(b - a) * WC, ncclFloat32, q, c->nccl, s);
-            }
-            ncclResult_t r2e = api->GroupEnd();
-            if (r != ncclSuccess || r2e != ncclSuccess)
-                st = set_error(RODINIA_E_NCCL, "srad_dist: cone broadcast failed");
-        } else if (st == RODINIA_OK) {
-            for (size_t i = 0; i < sl.size(); ++i) {
-                const int64_t q0 = sl[i].row0, qn = sl[i].own;
-                const int64_t a = std::max(q0, wr0), b = std::min(q0 + qn, wr1);
-                if (a >= b) continue;
-                const float* src = (c->kind == 1 ? ((float* const*)J_local)[i] : (float*)J_local);
-                cudaMemcpy2DAsync(W + (size_t)(a - wr0) * WC, WC * sizeof(float), src + (size_t)(a - q0) * C + wc0,
+    float* W = sc.W;
+    NcclApi* api = nullptr;
+    if (c->kind == 0 && c->nranks > 1) st = nccl_api(&api);
+    if (st == RODINIA_OK && api) {
+        ncclResult_t r = api->GroupStart();
+        for (int q = 0; q < c->nranks && r == ncclSuccess; ++q) {
+            int64_t q0, qn;
+            slab_of(R, c->nranks, q, &q0, &qn);
+            const int64_t a = std::max(q0, wr0), b = std::min(q0 + qn, wr1);
+            if (a >= b) continue;
+            float* part = W + (size_t)(a - wr0) * WC;
+            if (q == c->rank)  // owner packs its rows of the window
+                cudaMemcpy2DAsync(part, WC * sizeof(float), (const float*)J_local + (size_t)(a - q0) * C + wc0,
                                   rowb, WC * sizeof(float), (size_t)(b - a), cudaMemcpyDeviceToDevice, s);
-            }
+            r = api->Bcast(part, part, (size_t)(b - a) * WC, ncclFloat32, q, c->nccl, s);
+        }
+        ncclResult_t r2e = api->GroupEnd();
+        if (r != ncclSuccess || r2e != ncclSuccess)
+            st = set_error(RODINIA_E_NCCL, "srad_dist: cone broadcast failed");
+    } else if (st == RODINIA_OK) {
+        for (size_t i = 0; i < sl.size(); ++i) {
+            const int64_t q0 = sl[i].row0, qn = sl[i].own;
+            const int64_t a = std::max(q0, wr0), b = std::min(q0 + qn, wr1);
+            if (a >= b) continue;
+            const float* src = (c->kind == 1 ? ((float* const*)J_local)[i] : (float*)J_local);
+            cudaMemcpy2DAsync(W + (size_t)(a - wr0) * WC, WC * sizeof(float), src + (size_t)(a - q0) * C + wc0,
+                              rowb, WC * sizeof(float), (size_t)(b - a), cudaMemcpyDeviceToDevice, s);
         }
     }
     if (st == RODINIA_OK)
-        srad::engine_steps(&we, W, we.jb, 0, niter, true, (int)(r1 - wr0), (int)(c1 - wc0), (int)(r2 - r1 + 1),
+        srad::engine_steps(&sc.we, W, sc.we.jb, 0, niter, true, (int)(r1 - wr0), (int)(c1 - wc0), (int)(r2 - r1 + 1),
                            (int)(c2 - c1 + 1), 0.25f * lambda, s);
 
     // ---- slabs: halo D above, 2D below, exchange every D iterations
-    std::vector<srad::Engine> eng(sl.size());
     for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
         Slab& x = sl[i];
-        st = scratch_alloc((void**)&x.buf[0], (size_t)x.rows() * rowb, s);
-        if (st == RODINIA_OK) st = srad::engine_alloc(&eng[i], p, x.rows(), (int)C, niter, s);
-        if (st == RODINIA_OK) {
-            x.buf[1] = eng[i].jb;
-            const float* src = (c->kind == 1 ? ((float* const*)J_local)[i] : (float*)J_local);
-            cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, src, x.own * rowb, cudaMemcpyDeviceToDevice, s);
-            cudaMemcpyAsync(eng[i].its, we.its, (size_t)niter * sizeof(SradIter), cudaMemcpyDeviceToDevice, s);
-        }
+        const float* src = (c->kind == 1 ? ((float* const*)J_local)[i] : (float*)J_local);
+        if (cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, src, x.own * rowb, cudaMemcpyDeviceToDevice, s) != cudaSuccess ||
+            cudaMemcpyAsync(sc.eng[i].its, sc.we.its, (size_t)niter * sizeof(SradIter), cudaMemcpyDeviceToDevice, s) !=
+                cudaSuccess)
+            st = cuda_error(cudaGetLastError(), "srad_dist copy-in", __FILE__, __LINE__);
     }
     std::vector<float*> cur(sl.size()), oth(sl.size());
     for (size_t i = 0; i < sl.size(); ++i) { cur[i] = sl[i].buf[0]; oth[i] = sl[i].buf[1]; }
@@ -433,7 +674,7 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
             st = exchange(c, sl, which, (int)C, 2 * D, D, false, s);
         }
         for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
-            float* res = srad::engine_steps(&eng[i], cur[i], oth[i], it, std::min(niter, it + D), false, 0, 0, 1, 1,
+            float* res = srad::engine_steps(&sc.eng[i], cur[i], oth[i], it, std::min(niter, it + D), false, 0, 0, 1, 1,
                                             0.25f * lambda, s);
             oth[i] = (res == cur[i]) ? oth[i] : cur[i];
             cur[i] = res;
@@ -445,12 +686,10 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
         if (cudaMemcpyAsync(dst, cur[i] + (size_t)x.top * C, x.own * rowb, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
             st = cuda_error(cudaGetLastError(), "srad_dist copy-out", __FILE__, __LINE__);
     }
-    if (st == RODINIA_OK && cudaGetLastError() != cudaSuccess) st = set_error(RODINIA_E_CUDA, "srad_dist: launch failed");
-    for (size_t i = 0; i < sl.size(); ++i) {
-        scratch_free(sl[i].buf[0], s);
-        srad::engine_free(&eng[i], s);
+    if (cudaEventRecord(c->ev_done, s) == cudaSuccess) c->done_recorded = true;
+    if (st == RODINIA_OK) {
+        const cudaError_t ce = cudaGetLastError();
+        if (ce != cudaSuccess) st = cuda_error(ce, "srad_dist", __FILE__, __LINE__);
     }
-    srad::engine_free(&we, s);
-    scratch_free(W, s);
     return st;
 }

@@ -42,6 +42,30 @@ def slab(global_rows: int, nranks: int, rank: int):
     return r0.value, n.value
 
 
+class DistPlan(ctypes.Structure):
+    """rodinia_dist_plan: the schedule one rank follows (rodinia_dist_schedule)."""
+    _fields_ = [("row0", ctypes.c_int64), ("own", ctypes.c_int64), ("top", ctypes.c_int32),
+                ("bot", ctypes.c_int32), ("period", ctypes.c_int32), ("send_up", ctypes.c_int32),
+                ("send_down", ctypes.c_int32), ("exchanges", ctypes.c_int32), ("overlap", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("cone_r0", ctypes.c_int64), ("cone_r1", ctypes.c_int64),
+                ("cone_c0", ctypes.c_int64), ("cone_c1", ctypes.c_int64)]
+
+    def asdict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
+
+
+def schedule(kernel, global_rows: int, cols: int, nranks: int, rank: int, iterations: int,
+             roi=(0, 0, 0, 0), g=None) -> dict:
+    """Host-only: the slab, halo depths, exchange period/sizes and (srad) ROI-cone window the
+    library uses for `rank` (no device needed)."""
+    from . import _kernel
+    out = DistPlan()
+    r1, r2, c1, c2 = roi
+    check(lib.rodinia_dist_schedule(_kernel(kernel), global_rows, cols, nranks, rank, int(iterations),
+                                    r1, r2, c1, c2, _g(g), ctypes.byref(out)), "rodinia_dist_schedule")
+    return out.asdict()
+
+
 class HaloComm:
     def __init__(self, handle, nranks: int, rank: int, local: bool):
         self.handle = handle

@@ -2,11 +2,13 @@
 
 (a) bootstrap: rank 0 creates the NCCL unique id through the library, torch.distributed ships
     it, both ranks hold the same 128 bytes (what rodinia_comm_init consumes);
-(b) the decomposition protocol of csrc/dist.cu -- slab partition (rodinia_slab), halo depths
-    (hotspot D/D, srad D above / 2D below), exchange schedule (first rows up, last rows down,
-    every D steps), clamping at buffer edges, srad q0sqr(t) from the ROI dependency cone --
-    replayed with the CPU oracle as the per-slab solver and gloo send/recv as the transport:
-    the gathered result must equal the single-grid oracle bit for bit.
+(b) the decomposition csrc/dist.cu executes, taken from the library itself: every rank asks
+    rodinia_dist_schedule (host-only C ABI) for its slab, halo depths, exchange period and
+    sizes, overlap split and (srad) ROI-cone window, and runs exactly that schedule with the CPU
+    oracle as the per-slab solver and gloo send/recv as the transport -- including the hotspot
+    overlap split (interior from the owned rows alone, boundary strips of D halo + 2D owned
+    rows).  The gathered result must equal the single-grid oracle bit for bit, for several
+    temporal depths D and a rank count that does not divide the rows.
 """
 import os
 import socket
@@ -68,47 +70,73 @@ def _worker(rank, ws, port, q):
         dist.all_gather_object(ids, obj[0])
         assert len(ids[0]) == 128 and all(i == ids[0] for i in ids)
 
-        # (b1) hotspot: halo D = steps per exchange, iterations not a multiple of D
-        R, C, iters, D = 37, 23, 11, 3
+        # (b1) hotspot: the library's schedule for D = 1, 2, 3 (iterations not a multiple of D)
+        R, C, iters = 37, 23, 11
         T, P = synth.hotspot_inputs(R, C)
         cf = oracle.hotspot_coeffs_rodinia(512, 512)
-        r0, own = rg.dist.slab(R, ws, rank)
-        top = D if rank > 0 else 0
-        bot = D if rank + 1 < ws else 0
-        buf = np.zeros((top + own + bot, C))
-        pw = np.zeros_like(buf)
-        buf[top:top + own] = T[r0:r0 + own]
-        pw[top:top + own] = P[r0:r0 + own]
-        _exchange(pw, top, own, bot, D, D, rank, ws)
-        done = 0
-        while done < iters:
-            steps = min(D, iters - done)
-            _exchange(buf, top, own, bot, D, D, rank, ws)
-            buf = oracle.hotspot(buf, pw, steps, **cf)   # clamps at the buffer edges
-            done += steps
-        full = _gather_rows(buf[top:top + own], ws)
-        assert np.array_equal(full, oracle.hotspot(T, P, iters, **cf))
+        for D in (1, 2, 3):
+            g = (1, 1, 1, 1, 1, 0, 0) if D == 1 else (4, 1, 1, 1, D, 1, rg.RODINIA_STREAM)
+            if D == 3:
+                g = (2, 1, 1, 1, 4, 1, rg.RODINIA_STREAM)  # h = 4
+            pl = rg.dist.schedule("hotspot", R, C, ws, rank, iters, g=g)
+            D = pl["period"]
+            r0, own, top, bot = pl["row0"], pl["own"], pl["top"], pl["bot"]
+            assert (r0, own) == rg.dist.slab(R, ws, rank)
+            buf = np.zeros((top + own + bot, C))
+            pw = np.zeros_like(buf)
+            buf[top:top + own] = T[r0:r0 + own]
+            pw[top:top + own] = P[r0:r0 + own]
+            _exchange(pw, top, own, bot, pl["send_up"] or D, pl["send_down"] or D, rank, ws)
+            done = nex = 0
+            while done < iters:
+                steps = min(D, iters - done)
+                _exchange(buf, top, own, bot, pl["send_up"] or D, pl["send_down"] or D, rank, ws)
+                nex += 1
+                if pl["overlap"] and steps == D:
+                    # interior: owned rows only -> rows [D, own - D) exact
+                    inner = oracle.hotspot(buf[top:top + own], pw[top:top + own], steps, **cf)
+                    new = np.zeros_like(buf)
+                    new[top + D:top + own - D] = inner[D:own - D]
+                    ts = oracle.hotspot(buf[:top + 2 * D], pw[:top + 2 * D], steps, **cf)
+                    new[top:top + D] = ts[top:top + D]
+                    b0 = top + own - 2 * D
+                    bs = oracle.hotspot(buf[b0:], pw[b0:], steps, **cf)
+                    new[top + own - D:top + own] = bs[D:2 * D]
+                    buf = new
+                else:
+                    buf = oracle.hotspot(buf, pw, steps, **cf)   # clamps at the buffer edges
+                done += steps
+            assert nex == pl["exchanges"]
+            full = _gather_rows(buf[top:top + own], ws)
+            assert np.array_equal(full, oracle.hotspot(T, P, iters, **cf)), D
 
-        # (b2) srad: halo D above, 2D below; q0sqr(t) from the ROI cone window
-        R, C, n, D, lam = 41, 30, 7, 1, 0.5
+        # (b2) srad: the library's schedule (halo D above, 2D below, exchange every D iterations)
+        # and its ROI-cone window for q0sqr(t)
+        R, C, n, lam = 41, 30, 7, 0.5
         r1, r2, c1, c2 = 25, 33, 4, 12           # ROI owned by rank 1, read by both
         J = synth.srad_input(R, C)
-        w = J[max(0, r1 - n):min(R, r2 + 2 * n + 3), max(0, c1 - n):min(C, c2 + 2 * n + 3)]
-        _, q0 = oracle.srad(w, r1 - max(0, r1 - n), r2 - max(0, r1 - n), c1 - max(0, c1 - n),
-                            c2 - max(0, c1 - n), lam, n, return_q0=True)
         _, q0_full = oracle.srad(J, r1, r2, c1, c2, lam, n, return_q0=True)
-        assert np.array_equal(q0, q0_full)       # the cone reproduces q0sqr(t) exactly
+        ref = oracle.srad(J, r1, r2, c1, c2, lam, n)
+        for Dg in (1, 2, 3, 0):
+            g = None if Dg == 0 else (4, 1, 1, 2, Dg, 1, rg.RODINIA_STREAM)
+            pl = rg.dist.schedule("srad", R, C, ws, rank, n, roi=(r1, r2, c1, c2), g=g)
+            D = pl["period"]
+            assert pl["top"] in (0, D) and pl["bot"] in (0, 2 * D)
+            w0, w1, v0, v1 = pl["cone_r0"], pl["cone_r1"], pl["cone_c0"], pl["cone_c1"]
+            _, q0 = oracle.srad(J[w0:w1, v0:v1], r1 - w0, r2 - w0, c1 - v0, c2 - v0, lam, n, return_q0=True)
+            assert np.array_equal(q0, q0_full)       # the cone reproduces q0sqr(t) exactly
+            r0, own, top, bot = pl["row0"], pl["own"], pl["top"], pl["bot"]
+            buf = np.zeros((top + own + bot, C))
+            buf[top:top + own] = J[r0:r0 + own]
+            for t in range(0, n, D):
+                _exchange(buf, top, own, bot, 2 * D, D, rank, ws)
+                for k in range(t, min(n, t + D)):
+                    buf = oracle.srad_step(buf, q0[k], lam)
+            full = _gather_rows(buf[top:top + own], ws)
+            assert np.array_equal(full, ref), Dg
+        D = 1
         r0, own = rg.dist.slab(R, ws, rank)
-        top = D if rank > 0 else 0
-        bot = 2 * D if rank + 1 < ws else 0
-        buf = np.zeros((top + own + bot, C))
-        buf[top:top + own] = J[r0:r0 + own]
-        for t in range(0, n, D):
-            _exchange(buf, top, own, bot, 2 * D, D, rank, ws)
-            for k in range(t, min(n, t + D)):
-                buf = oracle.srad_step(buf, q0[k], lam)
-        full = _gather_rows(buf[top:top + own], ws)
-        assert np.array_equal(full, oracle.srad(J, r1, r2, c1, c2, lam, n))
+        q0 = q0_full
 
         # negative control: srad with only D rows below is NOT equal (the 2-row reach)
         top, bot = (D if rank > 0 else 0), (D if rank + 1 < ws else 0)

@@ -103,3 +103,55 @@ def test_nccl_single_rank(rg):
     rg.rodinia_srad(J2, 0, 20, 0, 20, 0.5, 5)
     assert torch.equal(J, J2)
     comm.close()
+
+
+@pytest.mark.parametrize("P", [2, 3, 5, 8])
+def test_srad_local_slabs_temporal_depth(rg, P):
+    # halo D above / 2D below exchanged every D iterations; C % 4 == 0 while the
+    # ROI-cone window is 77 or 73 columns wide at a column offset that is not a multiple of 4
+    # (the window's fp64 ROI reduction must match the full grid's bit for bit)
+    R, C, n = 203, 96, 12
+    J = synth.srad_input(R, C)
+    comm = rg.dist.HaloComm.local_slabs(P)
+    for roi in [(100, 140, 5, 50), (0, 20, 30, 45)]:
+        for kern in [(4, 1, 1, 2), (1, 1, 2, 1)]:
+            for D in (1, 2, 4, 8):
+                g = (kern[0], kern[1], kern[2], kern[3], D, 1, rg.RODINIA_STREAM if kern[0] == 4 else 0)
+                g1 = g[:4] + (1,) + g[5:]
+                ref = torch.from_numpy(J).cuda()
+                rg.rodinia_srad(ref, *roi, 0.5, n, g=g1)
+                js = _split(rg, torch.from_numpy(J).cuda(), P)
+                comm.srad(js, R, *roi, 0.5, n, g=g)
+                torch.cuda.synchronize()
+                assert torch.equal(torch.cat(js), ref), (P, roi, g)
+    comm.close()
+
+
+def test_dist_buffers_reused_across_calls_and_streams(rg):
+    # the communicator keeps its slab buffers; calls of different shapes and on different
+    # streams stay bitwise equal to the single-GPU call (each call is ordered after the last)
+    comm = rg.dist.HaloComm.local_slabs(4)
+    c = rg.rodinia_hotspot_coeffs_rodinia(512, 512)
+    g = (4, 1, 1, 2, 8, 1, 2)
+    for (R, C, it) in [(300, 256, 17), (300, 256, 16), (190, 384, 9), (300, 256, 24)]:
+        T, Pw = synth.hotspot_inputs(R, C, seed_t=R, seed_p=C)
+        t, p = torch.from_numpy(T).cuda(), torch.from_numpy(Pw).cuda()
+        ref = rg.rodinia_hotspot(t, p, it, coeffs=c, g=g)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            ts, ps = _split(rg, t, 4), _split(rg, p, 4)
+            outs = [torch.empty_like(x) for x in ts]
+            comm.hotspot(ts, ps, outs, R, it, coeffs=c, g=g, stream=s)
+        torch.cuda.synchronize()
+        assert torch.equal(torch.cat(outs), ref), (R, C, it)
+    comm.close()
+
+
+def test_dist_schedule_matches_layout(rg):
+    # the host-side schedule the library follows (rodinia_dist_schedule)
+    pl = rg.dist.schedule("hotspot", 16384, 16384, 8, 3, 1000, g=(4, 1, 1, 8, 8, 1, 2 | (10 << 8)))
+    assert (pl["top"], pl["bot"], pl["period"], pl["send_up"], pl["send_down"], pl["exchanges"], pl["overlap"]) == \
+        (8, 8, 8, 8, 8, 125, 1)
+    pl = rg.dist.schedule("srad", 8192, 8192, 8, 0, 100, roi=(0, 127, 0, 127))
+    assert (pl["top"], pl["bot"], pl["period"], pl["send_up"], pl["send_down"]) == (0, 16, 8, 0, 8)
+    assert (pl["cone_r0"], pl["cone_r1"], pl["cone_c0"], pl["cone_c1"]) == (0, 330, 0, 330)

@@ -72,14 +72,15 @@ def _direct_grans():
 
 
 def _stream_grans(rg):
-    # every instantiated stream variant that survives the compile-time filter
+    # every instantiated stream variant; the ptxas-pruned (spilling) ones through RODINIA_FORCE
     out = []
     for r in rg.rodinia_variants("hotspot"):
         g = r["g"]
-        if not (g[6] & rg.RODINIA_STREAM) or r["status"] != 0:
+        if not (g[6] & rg.RODINIA_STREAM):
             continue
+        fl = g[6] | (rg.RODINIA_FORCE if r["status"] != 0 else 0)
         for bx, by in [(1, 1), (3, 2), (2, 16)]:
-            out.append((g[0], 1, bx, by, g[4], 1, g[6]))
+            out.append((g[0], 1, bx, by, g[4], 1, fl))
     return out
 
 

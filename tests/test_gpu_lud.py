@@ -84,7 +84,8 @@ def test_all_variants_bit_identical(rg):
             g = r["g"]
             stream = bool(g[6] & rg.RODINIA_STREAM)
             for bx, by in ([(1, 1), (1, 5)] if stream else [(1, 1), (2, 1), (7, 3)]):
-                gg = (g[0], g[1], bx, by, 1, g[5], g[6])
+                # RODINIA_FORCE: the ptxas-pruned (spilling) instantiations must agree bitwise too
+                gg = (g[0], g[1], bx, by, 1, g[5], g[6] | rg.RODINIA_FORCE)
                 try:
                     got = _lu(rg, A, panel, gg).cpu().numpy()
                 except rg.RodiniaError as e:
