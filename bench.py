@@ -128,19 +128,55 @@ def _barrier(ws):
 
 
 # ----------------------------------------------------------------------------- CPU reference
-def cpu_oracle_hotspot(rows_sample: int, cols: int, iters: int, N: int):
-    """Time the fp64 C oracle on a bounded sample (rows_sample x cols, `iters` steps)."""
+def host_cpu():
+    """The GPU box's host CPU as the CPU baseline runs on it (os.cpu_count() and lscpu)."""
+    info = {"cpu_count": os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            k, _, v = ln.partition(":")
+            if k.strip() in ("Model name", "CPU(s)", "Thread(s) per core", "Core(s) per socket", "Socket(s)",
+                             "L3 cache", "NUMA node(s)"):
+                info[k.strip()] = v.strip()
+    except Exception:  # noqa: BLE001
+        pass
+    return info
+
+
+def cpu_oracle_hotspot(rows_sample: int, cols: int, iters: int, N: int, threads: int = 1):
+    """Time the fp64 C oracle on a bounded sample (rows_sample x cols, `iters` steps) with
+    `threads` OpenMP threads (1 = the single-threaded build; 0 = all host cores)."""
     import numpy as np
 
     import oracle
     import synth
+    used = oracle.set_threads(threads)
     T, P = synth.hotspot_inputs(rows_sample, cols)
     c = oracle.hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6)
     T64, P64 = T.astype(np.float64), P.astype(np.float64)
     t0 = time.perf_counter()
     oracle.hotspot(T64, P64, iters, **c)
     dt = time.perf_counter() - t0
-    return rows_sample * cols * iters / dt, dt
+    oracle.set_threads(1)
+    return rows_sample * cols * iters / dt, dt, used
+
+
+def cpu_baseline_hotspot(N: int, target_s: float = 12.0):
+    """CPU oracle on a 1024-row sample of the N x N grid: OpenMP over all host cores (the
+    reported value) and the single-threaded build beside it."""
+    rows = 1024
+    cpu_oracle_hotspot(rows, N, 1, N, threads=0)  # warm-up (library load, page faults)
+    _, d1, _ = cpu_oracle_hotspot(rows, N, 1, N, threads=0)
+    it = max(1, min(200, int(round(target_s / max(d1, 1e-3)))))
+    rate, dt, used = cpu_oracle_hotspot(rows, N, it, N, threads=0)
+    _, d1s, _ = cpu_oracle_hotspot(rows, N, 1, N, threads=1)
+    its = max(1, min(40, int(round(0.3 * target_s / max(d1s, 1e-3)))))
+    rate1, dt1, _ = cpu_oracle_hotspot(rows, N, its, N, threads=1)
+    return {"value": rate, "unit": "cell-updates/s", "cores": used, "kind": "oracle",
+            "sample": f"{rows}x{N} rows x cols of the {N}x{N} grid, {it} iterations ({dt:.1f} s), fp64 plain C, "
+                      f"OpenMP over {used} threads (os.cpu_count() = {os.cpu_count()})",
+            "single_thread": {"value": rate1, "cores": 1, "sample": f"{rows}x{N}, {its} iterations ({dt1:.1f} s)"},
+            "host": host_cpu()}
 
 
 def run_reference(args):
@@ -149,17 +185,19 @@ def run_reference(args):
         return 0
     N, iters_full = args.rows, args.iters
     rows_sample = 1024
-    rate0, dt0 = cpu_oracle_hotspot(rows_sample, N, 1, N)  # calibration
-    it = max(1, min(50, int(round(6.0 / max(dt0, 1e-3)))))  # ~6 s per step
+    rate0, dt0, _ = cpu_oracle_hotspot(rows_sample, N, 1, N, threads=0)  # calibration
+    it = max(1, min(200, int(round(8.0 / max(dt0, 1e-3)))))  # ~8 s per step
     for _ in range(args.warmup):
-        cpu_oracle_hotspot(rows_sample, N, max(1, it // 4), N)
+        cpu_oracle_hotspot(rows_sample, N, max(1, it // 8), N, threads=0)
     rates, times = [], []
+    used = 1
     for _ in range(args.steps):
-        r, dt = cpu_oracle_hotspot(rows_sample, N, it, N)
+        r, dt, used = cpu_oracle_hotspot(rows_sample, N, it, N, threads=0)
         rates.append(r)
         times.append(dt)
     v = statistics.median(rates)
-    sample = f"{rows_sample}x{N} rows x cols, {it} iterations per step (of the {N}x{N}x{iters_full} workload), fp64 plain C"
+    sample = (f"{rows_sample}x{N} rows x cols, {it} iterations per step (of the {N}x{N}x{iters_full} workload), "
+              f"fp64 plain C, OpenMP over {used} threads")
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "cell-updates/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
@@ -167,8 +205,8 @@ def run_reference(args):
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"hotspot {N}x{N} fp32, {iters_full} iterations (CPU oracle sample)",
                    "rows": N, "cols": N, "iterations": iters_full},
-        "cpu_baseline": {"value": v, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
-                         "sample": sample},
+        "cpu_baseline": {"value": v, "unit": "cell-updates/s", "cores": used, "kind": "oracle",
+                         "sample": sample, "host": host_cpu()},
         "e2e": {"value": v, "unit": "cell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -194,28 +232,42 @@ def _time_steps(fn, steps, warmup, stream, on_start=None):
 
 
 def _cpu_srad(n):
-    """fp64 C oracle on a 512-row sample of the n x n image, 20 iterations (cell-updates/s)."""
+    """fp64 C oracle on a 512-row sample of the n x n image (cell-updates/s), all host cores
+    (OpenMP over the per-cell passes; the ROI sums stay sequential) and one thread."""
     import oracle
     import synth
     J = synth.srad_input(512, n)
-    t0 = time.perf_counter()
-    oracle.srad(J, 0, 127, 0, 127, 0.5, 20)
-    dt = time.perf_counter() - t0
-    return {"value": 512 * n * 20 / dt, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
-            "sample": f"512x{n} rows x cols, 20 iterations ({dt:.1f} s), fp64 plain C"}
+    out = {}
+    for thr, it in ((0, 40), (1, 10)):
+        used = oracle.set_threads(thr)
+        t0 = time.perf_counter()
+        oracle.srad(J, 0, 127, 0, 127, 0.5, it)
+        dt = time.perf_counter() - t0
+        out[thr] = (512 * n * it / dt, dt, used, it)
+    oracle.set_threads(1)
+    v, dt, used, it = out[0]
+    return {"value": v, "unit": "cell-updates/s", "cores": used, "kind": "oracle",
+            "sample": f"512x{n} rows x cols, {it} iterations ({dt:.1f} s), fp64 plain C, OpenMP {used} threads",
+            "single_thread": {"value": out[1][0], "cores": 1}}
 
 
 def _cpu_pathfinder():
     import oracle
     import synth
     w = synth.pathfinder_wall(100, 100000)
-    reps, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < 2.0:
-        oracle.pathfinder(w)
-        reps += 1
-    dt = (time.perf_counter() - t0) / reps
-    return {"value": 99 * 100000 / dt, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
-            "sample": f"full 100x100000 problem, {reps} calls, {dt*1e3:.2f} ms/call, int32 plain C"}
+    res = {}
+    for thr in (0, 1):
+        used = oracle.set_threads(thr)
+        reps, t0 = 0, time.perf_counter()
+        while time.perf_counter() - t0 < 2.0:
+            oracle.pathfinder(w)
+            reps += 1
+        res[thr] = ((time.perf_counter() - t0) / reps, reps, used)
+    oracle.set_threads(1)
+    dt, reps, used = res[0]
+    return {"value": 99 * 100000 / dt, "unit": "cell-updates/s", "cores": used, "kind": "oracle",
+            "sample": f"full 100x100000 problem, {reps} calls, {dt*1e3:.2f} ms/call, int32 plain C, OpenMP {used} threads",
+            "single_thread": {"value": 99 * 100000 / res[1][0], "cores": 1}}
 
 
 def _cpu_lud():
@@ -319,19 +371,20 @@ def extra_workloads(rg, torch, tune: bool):
         out["hotspot3d"] = res
     except Exception as e:  # noqa: BLE001
         out["hotspot3d"] = {"error": str(e)[:200]}
-    # pathfinder 100 rows x 100000 cols int32, per-call time over batches
+    # pathfinder 100 rows x 100000 cols int32 (BASELINE configs[1]): per-call time over CUDA-graph
+    # batches of calls (PAPER.md:305 drops runs under 1e-4 s), tuned vs uncoarsened, and the
+    # thread-coarsening sweep t = 1..8: for every t the TDO's best (CTA width,
+    # family, pyramid height) with t cells per thread, L2-warm (the 40 MB wall stays in the
+    # 126 MB L2 across calls) and L2-cold (a 2 x L2 buffer is rewritten before every call inside
+    # the graph; the flush-only graph's time is subtracted).
     try:
         import synth
         w = torch.from_numpy(synth.pathfinder_wall(100, 100000)).cuda()
         r = torch.empty(100000, dtype=torch.int32, device="cuda")
-        res = {}
-        for name, g in (("uncoarsened", (1, 1, 1, 1, 20, 0, 0)), ("tuned", None)):
-            if name == "tuned" and tune:
-                g, _ = rg.rodinia_tune("pathfinder", 100, 100000, 1, reps=3)
-            # one call is ~10 us of GPU work: time a CUDA graph of `batch` calls so host-side
-            # launch overhead does not pollute the per-call device time (PAPER.md:305 drops
-            # runs under 1e-4 s for the same reason)
-            batch = 200
+        l2 = torch.cuda.get_device_properties(0).L2_cache_size
+        flush = torch.empty(2 * l2 // 4, dtype=torch.float32, device="cuda")
+
+        def per_call(g, batch=200, cold=False):
             rg.rodinia_pathfinder(w, g=g, out=r)
             gs = torch.cuda.Stream()
             gs.wait_stream(s)
@@ -339,12 +392,42 @@ def extra_workloads(rg, torch, tune: bool):
             with torch.cuda.stream(gs):
                 with torch.cuda.graph(graph, stream=gs):
                     for _ in range(batch):
+                        if cold:
+                            flush.fill_(1.0)
                         rg.rodinia_pathfinder(w, g=g, out=r)
             torch.cuda.synchronize()
             ms = timed(graph.replay) / batch
+            if cold:
+                fg = torch.cuda.CUDAGraph()
+                with torch.cuda.stream(gs):
+                    with torch.cuda.graph(fg, stream=gs):
+                        for _ in range(batch):
+                            flush.fill_(1.0)
+                torch.cuda.synchronize()
+                ms -= timed(fg.replay) / batch
+            return ms
+
+        res = {}
+        tune_rows = []
+        for name, g in (("uncoarsened", (1, 1, 1, 1, 20, 0, 0)), ("tuned", None)):
+            if name == "tuned" and tune:
+                g, tune_rows = rg.rodinia_tune("pathfinder", 100, 100000, 1, reps=3)
+            ms = per_call(g)
             res[name] = {"ms_per_call": ms, "cell_updates_per_s": 99 * 100000 / (ms * 1e-3),
+                         "ms_per_call_l2_cold": per_call(g, batch=50, cold=True),
                          "g": list(g.astuple()) if hasattr(g, "astuple") else list(g)}
         res["speedup"] = res["uncoarsened"]["ms_per_call"] / res["tuned"]["ms_per_call"]
+        sweep = []
+        for t in range(1, 9):
+            cand = [x for x in tune_rows if x["status"] == 0 and x["median_ms"] > 0 and x["g"][0] == t]
+            if not cand:
+                continue
+            gt = min(cand, key=lambda x: x["median_ms"])["g"]
+            warm = per_call(gt)
+            cold = per_call(gt, batch=50, cold=True)
+            sweep.append({"t": t, "g": list(gt), "us_per_call_l2_warm": warm * 1e3, "us_per_call_l2_cold": cold * 1e3,
+                          "cell_updates_per_s_warm": 99 * 100000 / (warm * 1e-3)})
+        res["t_sweep"] = sweep
         # 4 B of wall per cell-update; the DP is latency-bound (99 dependent rows)
         hbm, src = _peaks()
         ach = 4.0 * res["tuned"]["cell_updates_per_s"] / 1e9
@@ -474,21 +557,25 @@ def run_ours(args):
     avg_launch_ms = _max_over_ranks(avg_launch_ms, ws)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
     traffic, traffic_src = None, None
-    # DRAM traffic per launch from the committed ncu --set full capture of the same kernel and
-    # granularity (profiles/<round>_hotspot.json), newest round first
+    # DRAM traffic per launch from a committed ncu --set full capture of the same kernel
+    # (profiles/<round>_hotspot.json): the exact benched granularity if captured, else the same
+    # instantiation (V, H, register budget) at another chunk height, newest round first
     import glob
+    caps = []
     for tp in sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_hotspot.json")), reverse=True):
         try:
             with open(tp) as f:
                 prof = json.load(f)
             pg = prof.get("granularity") or []
-            # same instantiation (V, H); the chunk height changes the halo share only slightly
-            if pg[:1] == [g.thread_x] and pg[4:5] == [g.temporal] and prof.get("traffic_bytes_per_launch"):
-                traffic = prof["traffic_bytes_per_launch"] * (rows_local * N) / (16384 * 16384)
-                traffic_src = f"{os.path.basename(tp)} (granularity {pg})"
-                break
-        except Exception:
-            traffic = None
+            if prof.get("traffic_bytes_per_launch") and pg[:1] == [g.thread_x] and pg[4:5] == [g.temporal] \
+                    and pg[6:7] == [g.flags]:
+                caps.append((pg == list(g.astuple()), tp, pg, prof["traffic_bytes_per_launch"]))
+        except Exception:  # noqa: BLE001
+            pass
+    if caps:
+        exact, tp, pg, tb = sorted(caps, key=lambda c: not c[0])[0]
+        traffic = tb * (rows_local * N) / (16384 * 16384)
+        traffic_src = f"{os.path.basename(tp)} (granularity {pg}, {'exact' if exact else 'same instantiation'})"
     roof_hbm = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
             "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
             "kernel": "hs_stream" if g.flags & rg.RODINIA_STREAM else "hs_direct",
@@ -514,10 +601,10 @@ def run_ours(args):
             "kernel": roof_hbm["kernel"], "avg_launch_ms": avg_launch_ms,
             "updates_per_launch": rows_local * N * h, "frac_of_nominal_fp32": ach_tf / fp32_peak}
 
-    # ---- uncoarsened variant (same timed protocol, fewer steps)
+    # ---- uncoarsened variant (same timed protocol: 1 warm-up, 3 timed steps)
     unc_ms = None
     if not args.no_extra:
-        unc_ms = _max_over_ranks(_time_steps(lambda: step(UNC), 1, 1, stream), ws)
+        unc_ms = _max_over_ranks(_time_steps(lambda: step(UNC), 3, 1, stream), ws)
 
     # ---- e2e at N > 1: each rank copies its slab from pinned host memory, solves through the
     # row-slab API, copies its slab back; max over ranks
@@ -576,12 +663,7 @@ def run_ours(args):
         # ---- CPU oracle baseline (bounded sample)
         cpu = None
         if not args.no_cpu:
-            r1, d1 = cpu_oracle_hotspot(1024, N, 1, N)
-            it = max(1, min(40, int(round(12.0 / max(d1, 1e-3)))))
-            rate, dt = cpu_oracle_hotspot(1024, N, it, N)
-            cpu = {"value": rate, "unit": "cell-updates/s", "cores": 1, "kind": "oracle",
-                   "sample": f"1024x{N} rows x cols of the {N}x{N} grid, {it} iterations "
-                             f"({dt:.1f} s), fp64 plain C, single thread"}
+            cpu = cpu_baseline_hotspot(N)
         extra = extra_workloads(rg, torch, not args.no_tune) if (ws == 1 and not args.no_extra) else {}
         speedups = {"hotspot": (unc_ms / ms) if unc_ms else None}
         for k, v in extra.items():  # geomean over BASELINE's four workloads (srad_v1 reported aside)
@@ -590,6 +672,9 @@ def run_ours(args):
         sp = [x for x in speedups.values() if x]
         geomean = float(np.exp(np.mean(np.log(sp)))) if sp else None
         clocks = clk.summary()
+        sr = extra.get("srad", {}) if isinstance(extra, dict) else {}
+        pf = extra.get("pathfinder", {}) if isinstance(extra, dict) else {}
+        ld = extra.get("lud", {}) if isinstance(extra, dict) else {}
         result = {
             "metric": METRIC, "value": value, "unit": "cell-updates/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -602,19 +687,31 @@ def run_ours(args):
                        "parallelism": f"row-slab x{ws}" if ws > 1 else "single GPU",
                        "l2": "no flush: working set 3 GiB >> 126 MB L2",
                        "tune_seconds": round(t_tune, 1)},
-            "roofline": roof,
+            "workloads": extra,
+            "tuning": tuning,
             "roofline_hbm": roof_hbm,
+            "uncoarsened": {"ms_per_step": unc_ms, "steps": 3,
+                            "value": N * N * iters / (unc_ms * 1e-3) if unc_ms else None},
+            "speedup_vs_uncoarsened": speedups,
+            "paper_context": "27% Rodinia geomean speedup, A100/A4000, composite timing (PAPER.md:29)",
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches_timed,
             "clocks": clocks,
-            "uncoarsened": {"ms_per_step": unc_ms,
-                            "value": N * N * iters / (unc_ms * 1e-3) if unc_ms else None},
-            "speedup_vs_uncoarsened": speedups,
-            "geomean_speedup_vs_uncoarsened": geomean,
-            "workloads": extra,
-            "tuning": tuning,
-            "paper_context": "27% Rodinia geomean speedup, A100/A4000, composite timing (PAPER.md:29)",
+            "roofline": roof,
+            # the short summary last, so a tail of the line keeps it
+            "summary": {
+                "hotspot_cell_updates_per_s": value,
+                "hotspot_uncoarsened": N * N * iters / (unc_ms * 1e-3) if unc_ms else None,
+                "srad_cell_updates_per_s": (sr.get("tuned") or {}).get("cell_updates_per_s"),
+                "srad_hbm_frac": (sr.get("roofline") or {}).get("frac"),
+                "srad_v1_ms": ((extra.get("srad_v1") or {}).get("tuned") or {}).get("ms") if isinstance(extra, dict) else None,
+                "pathfinder_us_per_call": 1e3 * (pf.get("tuned") or {}).get("ms_per_call", float("nan")),
+                "lud_panel16_ms": (ld.get("tuned") or {}).get("ms"),
+                "lud_panel128_tc_ms": (ld.get("panel128_tc") or {}).get("ms"),
+                "geomean_speedup_vs_uncoarsened": geomean,
+                "cpu_oracle_all_cores": (cpu or {}).get("value"), "cpu_cores": (cpu or {}).get("cores"),
+            },
         }
         print(json.dumps(result), flush=True)
     if ws > 1:

@@ -419,7 +419,7 @@ static const StreamVariant kStream[] = {
     RG_HSS(4, 2, 16), RG_HSS(4, 2, 24),
     RG_HSS(4, 4, 12), RG_HSS(4, 4, 16), RG_HSS(4, 4, 20), RG_HSS(4, 4, 24),
     RG_HSS(4, 6, 10), RG_HSS(4, 6, 12), RG_HSS(4, 6, 16),
-    RG_HSS(4, 8, 8), RG_HSS(4, 8, 10), RG_HSS(4, 8, 12), RG_HSS(4, 8, 16),
+    RG_HSS(4, 8, 8), RG_HSS(4, 8, 10), RG_HSS(4, 8, 12), RG_HSS(4, 8, 14), RG_HSS(4, 8, 16),
     RG_HSS(2, 4, 16), RG_HSS(2, 4, 24), RG_HSS(2, 4, 32),
     RG_HSS(2, 8, 12), RG_HSS(2, 8, 16), RG_HSS(2, 8, 20), RG_HSS(2, 8, 24),
     RG_HSS(2, 12, 12), RG_HSS(2, 12, 16),
