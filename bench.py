@@ -167,7 +167,9 @@ def cpu_baseline_hotspot(N: int, target_s: float = 12.0):
     rows = 1024
     cpu_oracle_hotspot(rows, N, 1, N, threads=0)  # warm-up (library load, page faults)
     _, d1, _ = cpu_oracle_hotspot(rows, N, 1, N, threads=0)
-    it = max(1, min(200, int(round(target_s / max(d1, 1e-3)))))
+    _, d5, _ = cpu_oracle_hotspot(rows, N, 6, N, threads=0)
+    per = max((d5 - d1) / 5, 1e-4)  # per-iteration time without the per-call allocation
+    it = max(1, min(5000, int(round(target_s / per))))
     rate, dt, used = cpu_oracle_hotspot(rows, N, it, N, threads=0)
     _, d1s, _ = cpu_oracle_hotspot(rows, N, 1, N, threads=1)
     its = max(1, min(40, int(round(0.3 * target_s / max(d1s, 1e-3)))))
@@ -185,8 +187,11 @@ def run_reference(args):
         return 0
     N, iters_full = args.rows, args.iters
     rows_sample = 1024
-    rate0, dt0, _ = cpu_oracle_hotspot(rows_sample, N, 1, N, threads=0)  # calibration
-    it = max(1, min(200, int(round(8.0 / max(dt0, 1e-3)))))  # ~8 s per step
+    cpu_oracle_hotspot(rows_sample, N, 1, N, threads=0)  # warm-up
+    _, dt0, _ = cpu_oracle_hotspot(rows_sample, N, 1, N, threads=0)  # calibration
+    _, dt5, _ = cpu_oracle_hotspot(rows_sample, N, 6, N, threads=0)
+    per = max((dt5 - dt0) / 5, 1e-4)
+    it = max(1, min(5000, int(round(8.0 / per))))  # ~8 s per step
     for _ in range(args.warmup):
         cpu_oracle_hotspot(rows_sample, N, max(1, it // 8), N, threads=0)
     rates, times = [], []

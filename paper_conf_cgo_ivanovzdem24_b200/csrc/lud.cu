@@ -45,19 +45,7 @@ __global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, 
     const bool own = lane < r;
 #pragma unroll
     for (int j = 0; j < P; ++j) a[j] = (own && j < r) ? A[(size_t)(o + lane) * n + o + j] : 0.f;
-#pragma unroll
-    for (int kk = 0; kk < P - 1; ++kk) {
-        if (kk >= r - 1) break;  // uniform
-        const float piv = __shfl_sync(0xffffffffu, a[kk], kk);
-        const bool below = lane > kk && own;
-        const float l = __fdiv_rn(a[kk], piv);
-        if (below) a[kk] = l;
-#pragma unroll
-        for (int j = kk + 1; j < P; ++j) {
-            const float ukj = __shfl_sync(0xffffffffu, a[j], kk);
-            if (below) a[j] = __fsub_rn(a[j], __fmul_rn(l, ukj));
-        }
-    }
+    tc::diag_factor<P>(a, r, lane);
 #pragma unroll
     for (int j = 0; j < P; ++j)
         if (own && j < r) A[(size_t)(o + lane) * n + o + j] = a[j];
@@ -68,9 +56,17 @@ __global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, 
 // each own one column of U12 = L11^-1 A12 (forward substitution, unit-lower L11), lanes
 // P..2P-1 each own one row of L21 = A21 U11^-1.  Tiles are staged through shared memory with
 // coalesced loads, the substitutions run in registers with L11/U11 read by broadcast.
-template <int P>
-__global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
-    float* A = *slot;
+// Panel-128 path (IMG): the kernel also writes its U12 columns / L21 rows, as the hi/lo TF32
+// parts of the tensor-core operand images, into the outer block's images (rows / columns from
+// `base`, k index kap0 + i): the images tc_split would build from the same final values.
+struct PerimImg {
+    float* a;   // A image (L21 rows)
+    float* b;   // B image (U12 columns, K-major)
+    int base, kap0, ng;
+};
+
+template <int P, bool IMG>
+__device__ __forceinline__ void lud_perim_body(float* A, int n, int k, const PerimImg& im) {
     __shared__ float dia[P][P + 1], rowt[P][P + 1], colt[P][P + 1];
     const int o = k * P;
     const int tb = o + P * (blockIdx.x + 1);  // first row/col of this perimeter tile
@@ -94,9 +90,17 @@ __global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ sl
         for (int i = 1; i < P; ++i)
 #pragma unroll
             for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(dia[i][j], v[j]));
-        if (tx < w)
+        if (tx < w) {
 #pragma unroll
             for (int i = 0; i < P; ++i) A[(size_t)(o + i) * n + tb + tx] = v[i];
+            if constexpr (IMG) {
+#pragma unroll
+                for (int q = 0; q < P / 4; ++q) {
+                    const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
+                    tc::img_store4(im.b, im.ng, tb + tx - im.base, im.kap0 + 4 * q, f);
+                }
+            }
+        }
     } else {  // L21 row idx
         const int idx = tx - P;
 #pragma unroll
@@ -107,10 +111,27 @@ __global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ sl
             for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(v[j], dia[j][i]));
             v[i] = __fdiv_rn(v[i], dia[i][i]);
         }
-        if (idx < w)
+        if (idx < w) {
 #pragma unroll
             for (int i = 0; i < P; ++i) A[(size_t)(tb + idx) * n + o + i] = v[i];
+            if constexpr (IMG) {
+#pragma unroll
+                for (int q = 0; q < P / 4; ++q) {
+                    const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
+                    tc::img_store4(im.a, im.ng, tb + idx - im.base, im.kap0 + 4 * q, f);
+                }
+            }
+        }
     }
+}
+
+template <int P>
+__global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
+    lud_perim_body<P, false>(*slot, n, k, PerimImg{});
+}
+
+__global__ void __launch_bounds__(64) lud_perim_img(float* const* __restrict__ slot, int n, int k, PerimImg im) {
+    lud_perim_body<32, true>(*slot, n, k, im);
 }
 
 // ------------------------------------------------------------------ trailing update
@@ -360,33 +381,105 @@ __global__ void __launch_bounds__(256)
 }
 
 namespace tc {
-// Whole factorisation, 128-wide outer blocks (inner panel 32).  Returns the launch count.
-inline int launch_all(float* const* slot, int n, float* img_a, float* img_b, cudaStream_t s) {
+// Launch helpers for the captured panel-128 factorisation: every kernel of the latency chain
+// (diagonal, panel, restricted updates) carries the highest launch priority, so that in the
+// graph it is scheduled ahead of the concurrently running trailing GEMM's CTAs.
+struct Lnch {
+    cudaStream_t s;
+    int prio;   // cudaLaunchAttributePriority value (0 = default)
+};
+template <typename... KArgs, typename... Args>
+inline void launch_p(const Lnch& L, void (*fn)(KArgs...), dim3 grid, dim3 block, size_t smem, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = L.s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributePriority;
+    at[0].val.priority = L.prio;
+    cfg.attrs = at;
+    cfg.numAttrs = L.prio ? 1 : 0;
+    cudaLaunchKernelEx(&cfg, fn, (KArgs)args...);
+}
+
+inline int update_img(const Lnch& L, float* const* slot, int n, const Rect* rs, int nr, const Img& im, int diag0) {
+    Args a;
+    a.nrect = 0;
+    for (int i = 0; i < nr; ++i)
+        if (rs[i].m > 0 && rs[i].nn > 0 && rs[i].kk > 0) a.rect[a.nrect++] = rs[i];
+    if (a.nrect == 0) return 0;
+    if (a.nrect == 1) a.rect[1] = a.rect[0];
+    const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
+    launch_p(L, lud_tc_update2, dim3(grid), dim3(128), smem_bytes2(), slot, n, a, im, diag0);
+    return 1;
+}
+
+// Whole factorisation, 128-wide outer blocks (inner panel 32), with look-ahead.  Returns the
+// launch count.  imgs: 4 images of img_floats(n) floats (A and B for two outer blocks).
+//  main branch (cs, high priority), per outer block [o, e):
+//    for each inner panel p0 = o + 32j: lud_diag<32>; lud_perim_img (U12/L21 + their hi/lo
+//    operand images, K chunks 2j, 2j+1 of the block's image); the rank-32 update of the block's
+//    L-shaped panel region from those chunks;
+//    then the part of the rank-128 trailing update that the NEXT block's panel needs (rows
+//    [e, e2) x cols [e, n) and rows [e2, n) x cols [e, e2), e2 = e + 128), after the previous
+//    block's remainder update (same region of C);
+//  side branch (cs2): the remainder of the rank-128 update, rows/cols [e2, n), which runs
+//    concurrently with the next block's panel chain (disjoint parts of C; the images are
+//    double-buffered by block parity).
+inline int launch_all(float* const* slot, int n, float* const imgs[4], cudaStream_t cs, cudaStream_t cs2,
+                      cudaEvent_t ev_fork, cudaEvent_t ev_img, cudaEvent_t ev_rest, int prio_hi) {
     constexpr int NB = 128, P = 32;
     const int m32 = (n + P - 1) / P;
     int launches = 0;
-    for (int o = 0; o < n; o += NB) {
+    const Lnch H{cs, prio_hi}, S{cs2, 0};
+    cudaEventRecord(ev_fork, cs);
+    cudaStreamWaitEvent(cs2, ev_fork, 0);  // fork the side branch into the capture
+    bool rest_pending = false;
+    for (int o = 0, blk = 0; o < n; o += NB, ++blk) {
         const int e = std::min(n, o + NB);
+        const int base = std::min(o + P, n);
+        const int ng = ((n - base + 127) / 128 + 1) * 16;
+        float* ia = imgs[2 * (blk & 1)];
+        float* ib = imgs[2 * (blk & 1) + 1];
+        const Img im{ia, ib, base, base, ng, ng, 0};
         for (int k = o / P; k * P < e; ++k) {
-            lud_diag<P><<<1, 32, 0, s>>>(slot, n, k);
-            ++launches;
+            if (k == 0) {  // every later diagonal tile is factored by the update that precedes it
+                launch_p(H, lud_diag<P>, dim3(1), dim3(32), 0, slot, n, k);
+                ++launches;
+            }
             if (k == m32 - 1) break;
-            lud_perim<P><<<m32 - k - 1, 2 * P, 0, s>>>(slot, n, k);
+            const int j = k - o / P;
+            launch_p(H, lud_perim_img, dim3(m32 - k - 1), dim3(2 * P), 0, slot, n, k, PerimImg{ia, ib, base, P * j, ng});
             ++launches;
             const int p0 = k * P, a = p0 + P;  // inner panel columns [p0, a)
             if (a < e) {
                 // rank-32 update restricted to the outer block's L-shaped panel region
                 const Rect rs[2] = {make_rect(a, a, n - a, e - a, p0, P), make_rect(a, e, e - a, n - e, p0, P)};
-                launch_update2(slot, n, rs, 2, a, img_a, img_b, s);
-                launches += 3;
+                Img ij = im;
+                ij.c0 = 2 * j;
+                launches += update_img(H, slot, n, rs, 2, ij, a);  // + diagonal tile of step k+1
             }
         }
-        if (e < n) {  // rank-128 trailing update on the tensor cores
-            const Rect r = make_rect(e, e, n - e, n - e, o, e - o);
-            launch_update2(slot, n, &r, 1, e, img_a, img_b, s);
-            launches += 3;
+        if (e < n) {  // rank-128 trailing update on the tensor cores, split for look-ahead
+            const int e2 = std::min(n, e + NB);
+            cudaEventRecord(ev_img, cs);  // this block's images are complete
+            if (rest_pending) cudaStreamWaitEvent(cs, ev_rest, 0);
+            const Rect rs[2] = {make_rect(e, e, e2 - e, n - e, o, e - o), make_rect(e2, e, n - e2, e2 - e, o, e - o)};
+            launches += update_img(H, slot, n, rs, 2, im, e);  // + diagonal tile of the next block
+            if (e2 < n) {
+                cudaStreamWaitEvent(cs2, ev_img, 0);
+                const Rect rr = make_rect(e2, e2, n - e2, n - e2, o, e - o);
+                launches += update_img(S, slot, n, &rr, 1, im, -1);
+                cudaEventRecord(ev_rest, cs2);
+                rest_pending = true;
+            } else {
+                rest_pending = false;
+            }
         }
     }
+    cudaEventRecord(ev_rest, cs2);
+    cudaStreamWaitEvent(cs, ev_rest, 0);  // join
     return launches;
 }
 }  // namespace tc
@@ -536,19 +629,31 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         if (!ge.slot) RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
         const void* ifn = pl.tc ? (const void*)tc::lud_tc_update2
                                 : pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
-        if (pl.tc && !ge.img) RG_CUDA(cudaMalloc(&ge.img, 2 * tc::img_floats(n) * sizeof(float)));
+        if (pl.tc && !ge.img) RG_CUDA(cudaMalloc(&ge.img, 4 * tc::img_floats(n) * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
-        cudaStream_t cs;
+        cudaStream_t cs, cs2;
+        cudaEvent_t ev[3];
         RG_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+        RG_CUDA(cudaStreamCreateWithFlags(&cs2, cudaStreamNonBlocking));
+        for (auto& x : ev) RG_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
+        int prio_lo = 0, prio_hi = 0;
+        cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         cudaGraph_t graph;
         RG_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
         lud_set_slot<<<1, 1, 0, cs>>>(ge.slot, a);  // root node; argument replaced per launch
         int nl = 3 * m - 2;
-        if (pl.tc) nl = tc::launch_all(ge.slot, n, ge.img, ge.img + tc::img_floats(n), cs);
-        else launch_all(pl, ge.slot, n, cs);
+        if (pl.tc) {
+            const size_t f = tc::img_floats(n);
+            float* const imgs[4] = {ge.img, ge.img + f, ge.img + 2 * f, ge.img + 3 * f};
+            nl = tc::launch_all(ge.slot, n, imgs, cs, cs2, ev[0], ev[1], ev[2], prio_hi);
+        } else {
+            launch_all(pl, ge.slot, n, cs);
+        }
         cudaError_t e = cudaStreamEndCapture(cs, &graph);
         cudaStreamDestroy(cs);
+        cudaStreamDestroy(cs2);
+        for (auto& x : ev) cudaEventDestroy(x);
         if (e != cudaSuccess) return cuda_error(e, "lud graph capture", __FILE__, __LINE__);
         size_t nroot = 1;
         cudaGraphNode_t root = nullptr;

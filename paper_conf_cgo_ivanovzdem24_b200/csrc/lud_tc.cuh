@@ -74,6 +74,30 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
         "r"(parity));
 }
 
+// In-tile Doolittle of a P x P diagonal tile held one row per lane (a[j] = element (lane, j);
+// rows/columns >= r are ignored): step kk broadcasts row kk with warp shuffles and every lane
+// below it subtracts l_ik * u_kj.  Per element this is Doolittle's sequence (products
+// subtracted in ascending k, L divided by the pivot after its k < j terms) with separate
+// multiply and subtract as in Rodinia's lud_diagonal.  lud_diag and the panel-128 update's
+// fused diagonal both call this, so both give the same bits.
+template <int P>
+__device__ __forceinline__ void diag_factor(float (&a)[P], int r, int lane) {
+    const bool own = lane < r;
+#pragma unroll
+    for (int kk = 0; kk < P - 1; ++kk) {
+        if (kk >= r - 1) break;  // uniform
+        const float piv = __shfl_sync(0xffffffffu, a[kk], kk);
+        const bool below = lane > kk && own;
+        const float l = __fdiv_rn(a[kk], piv);
+        if (below) a[kk] = l;
+#pragma unroll
+        for (int j = kk + 1; j < P; ++j) {
+            const float ukj = __shfl_sync(0xffffffffu, a[j], kk);
+            if (below) a[j] = __fsub_rn(a[j], __fmul_rn(l, ukj));
+        }
+    }
+}
+
 __device__ __forceinline__ void split_tf32(float x, float& hi, float& lo) {
     hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
     lo = __fsub_rn(x, hi);
@@ -293,12 +317,29 @@ struct Img {
     const float* a;   // A image (rows from a_base)
     const float* b;   // B image (columns from b_base)
     int a_base, b_base, nga, ngb;
+    int c0;           // first K chunk of the image this update reads (chunks c0 .. c0+nchunks-1)
 };
+
+// Store 4 consecutive k values (kap % 4 == 0) of image row rho as hi/lo TF32 parts (the layout
+// above); used by tc_split and by the panel kernel that writes the images as it solves.
+__device__ __forceinline__ void img_store4(float* __restrict__ img, int ng, int rho, int kap, const float (&v)[4]) {
+    float4 h, l;
+    split_tf32(v[0], h.x, l.x); split_tf32(v[1], h.y, l.y);
+    split_tf32(v[2], h.z, l.z); split_tf32(v[3], h.w, l.w);
+    const int c = kap / KC2, kq = (kap % KC2) / 4, g = rho >> 3, rr = rho & 7;
+    *reinterpret_cast<float4*>(img + ((size_t)(c * 2) * ng + g) * (KC2 * 8) + kq * 32 + rr * 4) = h;
+    *reinterpret_cast<float4*>(img + ((size_t)(c * 2 + 1) * ng + g) * (KC2 * 8) + kq * 32 + rr * 4) = l;
+}
 
 // C -= A*B on 128 x 128 tiles: warp 0 lane 0 produces (bulk copies into an NS2-stage ring),
 // warp 1 lane 0 issues the 3xTF32 MMAs into TMEM and releases stages with tcgen05.commit; all
 // four warps run the epilogue (tcgen05.ld, C -= acc in place).
-__global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__ slot, int n, Args args, Img im) {
+// diag0 >= 0: the CTA whose tile starts at (diag0, diag0) also factors the 32 x 32 diagonal tile
+// of the next panel step (its warp 0 forms C - acc for that block in registers and runs
+// diag_factor instead of reducing it into C), which removes the separate lud_diag launch from
+// the factorisation's latency chain.
+__global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__ slot, int n, Args args, Img im,
+                                                      int diag0) {
     constexpr int PART = BM * KC2 * 4;
     constexpr int STAGE = 4 * PART;
     constexpr uint32_t SBO = KC2 * 32;
@@ -340,10 +381,11 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
             if (c >= NS2) mbar_wait(&empty[s], ((c / NS2) - 1) & 1);
             uint8_t* st = sm + s * STAGE;
             mbar_expect_tx(&full[s], STAGE);
-            const float* ah = im.a + ((size_t)(c * 2) * im.nga + ga) * (KC2 * 8);
-            const float* al = im.a + ((size_t)(c * 2 + 1) * im.nga + ga) * (KC2 * 8);
-            const float* bh = im.b + ((size_t)(c * 2) * im.ngb + gb) * (KC2 * 8);
-            const float* bl = im.b + ((size_t)(c * 2 + 1) * im.ngb + gb) * (KC2 * 8);
+            const int ci = c + im.c0;
+            const float* ah = im.a + ((size_t)(ci * 2) * im.nga + ga) * (KC2 * 8);
+            const float* al = im.a + ((size_t)(ci * 2 + 1) * im.nga + ga) * (KC2 * 8);
+            const float* bh = im.b + ((size_t)(ci * 2) * im.ngb + gb) * (KC2 * 8);
+            const float* bl = im.b + ((size_t)(ci * 2 + 1) * im.ngb + gb) * (KC2 * 8);
             bulk_g2s(st, ah, PART, &full[s]);
             bulk_g2s(st + PART, al, PART, &full[s]);
             bulk_g2s(st + 2 * PART, bh, PART, &full[s]);
@@ -378,6 +420,40 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
 
     const int r = row0 + warp * 32 + lane;
     const int ncols = min(BN, cend - col0);
+    const bool dtile = diag0 >= 0 && row0 == diag0 && col0 == diag0;  // this CTA owns the next diagonal tile
+    if (dtile && warp == 0) {
+        uint32_t v[32];
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+              "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+              "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+              "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+            : "r"(tmem));
+        asm volatile("tcgen05.wait::ld.sync.aligned;"
+                     : "+r"(v[0]), "+r"(v[1]), "+r"(v[2]), "+r"(v[3]), "+r"(v[4]), "+r"(v[5]), "+r"(v[6]),
+                       "+r"(v[7]), "+r"(v[8]), "+r"(v[9]), "+r"(v[10]), "+r"(v[11]), "+r"(v[12]), "+r"(v[13]),
+                       "+r"(v[14]), "+r"(v[15]), "+r"(v[16]), "+r"(v[17]), "+r"(v[18]), "+r"(v[19]),
+                       "+r"(v[20]), "+r"(v[21]), "+r"(v[22]), "+r"(v[23]), "+r"(v[24]), "+r"(v[25]),
+                       "+r"(v[26]), "+r"(v[27]), "+r"(v[28]), "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
+                     :
+                     : "memory");
+        const int rd = min(32, n - diag0);
+        float a[32];
+        const float* crow = A + (size_t)(diag0 + lane) * n + diag0;
+#pragma unroll
+        for (int j = 0; j < 32; ++j)  // C - acc of the diagonal block, as the epilogue would store it
+            a[j] = (lane < rd && j < rd) ? __fsub_rn(crow[j], __uint_as_float(v[j])) : 0.f;
+        diag_factor<32>(a, rd, lane);
+        if (lane < rd) {
+            float* wrow = A + (size_t)(diag0 + lane) * n + diag0;
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+                if (j < rd) wrow[j] = a[j];
+        }
+    }
     if (vec && (ncols & 3) == 0) {
         // Epilogue through the L2: -acc rows staged in the (now idle) pipeline shared memory,
         // then one bulk reduce-add (cp.reduce.async.bulk .add.f32) per row into C.  x + (-y) is
@@ -413,15 +489,16 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
         }
         // generic-proxy writes -> async proxy (bulk copy engine) reads
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        if (r < rend)
+        const int skip = (dtile && warp == 0) ? 32 : 0;  // the diagonal block was stored factored
+        if (r < rend && ncols > skip)
             asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
-                             A + (size_t)r * n + col0),
-                         "r"(smem_u32(row_s)), "r"(ncols * 4)
+                             A + (size_t)r * n + col0 + skip),
+                         "r"(smem_u32(row_s + skip * 4)), "r"((ncols - skip) * 4)
                          : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     } else
-    for (int jb = 0; jb < BN / 32; ++jb) {  // ragged or unaligned C: read-modify-write per row
+    for (int jb = (dtile && warp == 0) ? 1 : 0; jb < BN / 32; ++jb) {  // ragged or unaligned C: RMW per row
         uint32_t v[32];
         const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(jb * 32);
         asm volatile(
@@ -516,9 +593,9 @@ inline void launch_update2(float* const* slot, int n, const Rect* rs, int nr, in
     const int total = ng * 8 * nchunks * (KC2 / 4);
     const int grid_s = std::min((total + 255) / 256, 148 * 8);
     tc_split<<<dim3(grid_s, 2), 256, 0, s>>>(slot, n, img_a, img_b, base, k0, kk, ng, nchunks);
-    Img im{img_a, img_b, base, base, ng, ng};
+    Img im{img_a, img_b, base, base, ng, ng, 0};
     const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
-    lud_tc_update2<<<grid, 128, smem_bytes2(), s>>>(slot, n, a, im);
+    lud_tc_update2<<<grid, 128, smem_bytes2(), s>>>(slot, n, a, im, -1);
 }
 
 }  // namespace tc
