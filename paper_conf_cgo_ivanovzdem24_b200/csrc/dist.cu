@@ -68,6 +68,7 @@ struct rodinia_comm {
     cudaEvent_t ev_ready = nullptr, ev_strips = nullptr;
     cudaEvent_t ev_done = nullptr;        // end of the previous call (orders calls on any stream)
     bool done_recorded = false;
+    std::vector<cudaEvent_t> ev_cone;     // srad: q0sqr of exchange period p is ready
     // persistent buffers of the last shape (hotspot and srad separately)
     struct HsCache { int64_t R = 0, C = 0; int D = 0; std::vector<rg::Slab> sl; } hs;
     struct SrCache {
@@ -424,6 +425,8 @@ extern "C" rodinia_status rodinia_comm_destroy(rodinia_comm* c) {
             cudaEventDestroy(c->ev_ready);
             cudaEventDestroy(c->ev_strips);
             cudaEventDestroy(c->ev_done);
+            for (auto e : c->ev_cone) cudaEventDestroy(e);
+            c->ev_cone.clear();
             cudaGetLastError();  // teardown errors are not reported to later calls
         }
         if (c->kind == 0 && c->nccl) {
@@ -610,13 +613,14 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
             sc.sl.push_back(x);
         }
         sc.eng.resize(want.size());
-        for (size_t i = 0; i < want.size(); ++i) {
-            RG_TRY(srad::engine_alloc(&sc.eng[i], p, sc.sl[i].rows(), (int)C, niter, s));
-            sc.sl[i].buf[1] = sc.eng[i].jb;
-        }
         RG_TRY(dev_alloc(&sc.W, (size_t)WR * WC));
         RG_TRY(srad::engine_alloc(&sc.we, p, WR, WC, niter, s));
         sc.have_we = true;
+        for (size_t i = 0; i < want.size(); ++i) {
+            RG_TRY(srad::engine_alloc(&sc.eng[i], p, sc.sl[i].rows(), (int)C, niter, s));
+            sc.sl[i].buf[1] = sc.eng[i].jb;
+            sc.eng[i].its = sc.we.its;  // q0sqr(t) read from the cone engine's table (no copy)
+        }
         sc.R = R; sc.C = C; sc.D = D; sc.niter_cap = niter; sc.WR = WR; sc.WC = WC; sc.g = gg;
     }
     std::vector<Slab>& sl = sc.sl;
@@ -652,27 +656,48 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
                               rowb, WC * sizeof(float), (size_t)(b - a), cudaMemcpyDeviceToDevice, s);
         }
     }
-    if (st == RODINIA_OK)
-        srad::engine_steps(&sc.we, W, sc.we.jb, 0, niter, true, (int)(r1 - wr0), (int)(c1 - wc0), (int)(r2 - r1 + 1),
-                           (int)(c2 - c1 + 1), 0.25f * lambda, s);
+    // The cone's iterations (one statistics + one update launch each on a window of at most
+    // (3n)^2 cells: launch-latency bound) run on the side stream, one exchange period ahead of
+    // the slab iterations, which wait for period p's q0sqr values only (ev_cone[p]).  NCCL work
+    // stays on the compute stream.
+    const int nper = (niter + D - 1) / D;
+    while ((int)c->ev_cone.size() < nper) {
+        cudaEvent_t e;
+        RG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        c->ev_cone.push_back(e);
+    }
+    if (st == RODINIA_OK) {
+        RG_CUDA(cudaEventRecord(c->ev_ready, s));  // the window's J0 has been gathered
+        RG_CUDA(cudaStreamWaitEvent(c->side, c->ev_ready, 0));
+        float* wc = W;
+        float* wo = sc.we.jb;
+        for (int q = 0; q < nper; ++q) {
+            float* res = srad::engine_steps(&sc.we, wc, wo, q * D, std::min(niter, (q + 1) * D), true,
+                                            (int)(r1 - wr0), (int)(c1 - wc0), (int)(r2 - r1 + 1), (int)(c2 - c1 + 1),
+                                            0.25f * lambda, c->side);
+            wo = (res == wc) ? wo : wc;
+            wc = res;
+            RG_CUDA(cudaEventRecord(c->ev_cone[q], c->side));
+        }
+    }
 
     // ---- slabs: halo D above, 2D below, exchange every D iterations
     for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
         Slab& x = sl[i];
         const float* src = (c->kind == 1 ? ((float* const*)J_local)[i] : (float*)J_local);
-        if (cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, src, x.own * rowb, cudaMemcpyDeviceToDevice, s) != cudaSuccess ||
-            cudaMemcpyAsync(sc.eng[i].its, sc.we.its, (size_t)niter * sizeof(SradIter), cudaMemcpyDeviceToDevice, s) !=
-                cudaSuccess)
+        if (cudaMemcpyAsync(x.buf[0] + (size_t)x.top * C, src, x.own * rowb, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
             st = cuda_error(cudaGetLastError(), "srad_dist copy-in", __FILE__, __LINE__);
     }
     std::vector<float*> cur(sl.size()), oth(sl.size());
     for (size_t i = 0; i < sl.size(); ++i) { cur[i] = sl[i].buf[0]; oth[i] = sl[i].buf[1]; }
-    for (int it = 0; st == RODINIA_OK && it < niter; it += D) {
+    for (int it = 0, q = 0; st == RODINIA_OK && it < niter; it += D, ++q) {
         if (c->nranks > 1) {
             // exchange on whichever buffer currently holds J (same parity on every slab)
             const int which = (cur[0] == sl[0].buf[0]) ? 0 : 1;
             st = exchange(c, sl, which, (int)C, 2 * D, D, false, s);
         }
+        if (st == RODINIA_OK && cudaStreamWaitEvent(s, c->ev_cone[q], 0) != cudaSuccess)
+            st = cuda_error(cudaGetLastError(), "srad_dist cone wait", __FILE__, __LINE__);
         for (size_t i = 0; i < sl.size() && st == RODINIA_OK; ++i) {
             float* res = srad::engine_steps(&sc.eng[i], cur[i], oth[i], it, std::min(niter, it + D), false, 0, 0, 1, 1,
                                             0.25f * lambda, s);
