@@ -65,9 +65,17 @@ struct PerimImg {
     int base, kap0, ng;
 };
 
+// Threads [0, P) own the U12 columns (unit-lower solve with L11 = dia's strict lower part),
+// threads [P, 2P) the L21 rows (solve with U11, then divide by the pivot).  Both are the same
+// loop over a row-major matrix M (L11 itself, or U11 transposed) whose rows are read four at a
+// time with 128-bit shared loads; per element the subtractions run in ascending j exactly as in
+// the two separate loops this replaces (same bits), with half the code (the fully unrolled pair
+// of solves overflowed the instruction cache: "no instruction" was the top stall, ncu r02f).
 template <int P, bool IMG>
 __device__ __forceinline__ void lud_perim_body(float* A, int n, int k, const PerimImg& im) {
-    __shared__ float dia[P][P + 1], rowt[P][P + 1], colt[P][P + 1];
+    constexpr int LD = P + 4;  // 16-byte aligned rows
+    __shared__ __align__(16) float msm[2][P][LD];  // [0]: L11 = dia (row-major), [1]: U11^T
+    __shared__ float tile[2][P][P + 1];            // [0]: row tile A12, [1]: column tile A21
     const int o = k * P;
     const int tb = o + P * (blockIdx.x + 1);  // first row/col of this perimeter tile
     const int w = min(P, n - tb);             // its width (last tile may be partial)
@@ -77,49 +85,44 @@ __device__ __forceinline__ void lud_perim_body(float* A, int n, int k, const Per
 #pragma unroll
     for (int e0 = 0; e0 < P * P; e0 += 2 * P) {
         const int e = e0 + tx, i = e / P, j = e % P;
-        dia[i][j] = A[(size_t)(o + i) * n + o + j];
-        rowt[i][j] = j < w ? A[(size_t)(o + i) * n + tb + j] : 0.f;
-        colt[i][j] = i < w ? A[(size_t)(tb + i) * n + o + j] : 0.f;
+        const float d = A[(size_t)(o + i) * n + o + j];
+        msm[0][i][j] = d;
+        msm[1][j][i] = d;
+        tile[0][i][j] = j < w ? A[(size_t)(o + i) * n + tb + j] : 0.f;
+        tile[1][i][j] = i < w ? A[(size_t)(tb + i) * n + o + j] : 0.f;
     }
     __syncthreads();
+    const int half = tx / P, lane = tx - half * P;  // 0: U12 column `lane`, 1: L21 row `lane`
+    const float* M = &msm[half][0][0];
     float v[P];
-    if (tx < P) {  // U12 column tx
 #pragma unroll
-        for (int i = 0; i < P; ++i) v[i] = rowt[i][tx];
+    for (int i = 0; i < P; ++i) v[i] = half == 0 ? tile[0][i][lane] : tile[1][lane][i];
 #pragma unroll
-        for (int i = 1; i < P; ++i)
+    for (int i = 0; i < P; ++i) {
 #pragma unroll
-            for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(dia[i][j], v[j]));
-        if (tx < w) {
+        for (int jq = 0; jq < (i + 3) / 4; ++jq) {
+            const float4 m = *reinterpret_cast<const float4*>(M + i * LD + 4 * jq);
+            const float mm[4] = {m.x, m.y, m.z, m.w};
 #pragma unroll
-            for (int i = 0; i < P; ++i) A[(size_t)(o + i) * n + tb + tx] = v[i];
-            if constexpr (IMG) {
-#pragma unroll
-                for (int q = 0; q < P / 4; ++q) {
-                    const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
-                    tc::img_store4(im.b, im.ng, tb + tx - im.base, im.kap0 + 4 * q, f);
-                }
-            }
+            for (int t = 0; t < 4; ++t)
+                if (4 * jq + t < i) v[i] = __fsub_rn(v[i], __fmul_rn(mm[t], v[4 * jq + t < P ? 4 * jq + t : 0]));
         }
-    } else {  // L21 row idx
-        const int idx = tx - P;
+        if (half == 1) v[i] = __fdiv_rn(v[i], M[i * LD + i]);
+    }
+    if (lane < w) {
+        if (half == 0) {
 #pragma unroll
-        for (int i = 0; i < P; ++i) v[i] = colt[idx][i];
+            for (int i = 0; i < P; ++i) A[(size_t)(o + i) * n + tb + lane] = v[i];
+        } else {
 #pragma unroll
-        for (int i = 0; i < P; ++i) {
-#pragma unroll
-            for (int j = 0; j < i; ++j) v[i] = __fsub_rn(v[i], __fmul_rn(v[j], dia[j][i]));
-            v[i] = __fdiv_rn(v[i], dia[i][i]);
+            for (int i = 0; i < P; ++i) A[(size_t)(tb + lane) * n + o + i] = v[i];
         }
-        if (idx < w) {
+        if constexpr (IMG) {
+            float* img = half == 0 ? im.b : im.a;
 #pragma unroll
-            for (int i = 0; i < P; ++i) A[(size_t)(tb + idx) * n + o + i] = v[i];
-            if constexpr (IMG) {
-#pragma unroll
-                for (int q = 0; q < P / 4; ++q) {
-                    const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
-                    tc::img_store4(im.a, im.ng, tb + idx - im.base, im.kap0 + 4 * q, f);
-                }
+            for (int q = 0; q < P / 4; ++q) {
+                const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
+                tc::img_store4(img, im.ng, tb + lane - im.base, im.kap0 + 4 * q, f);
             }
         }
     }
