@@ -316,7 +316,7 @@ def extra_workloads(rg, torch, tune: bool):
         res = {}
         for name, g in (("uncoarsened", UNC), ("tuned", None)):
             if name == "tuned" and tune:
-                g, _ = rg.rodinia_tune("srad", n, n, it, reps=2)
+                g, _ = rg.rodinia_tune("srad", n, n, it, reps=5)
             ms = timed(lambda: (J.copy_(J0), rg.rodinia_srad(J, 0, 127, 0, 127, 0.5, it, g=g)))
             res[name] = {"ms": ms, "cell_updates_per_s": n * n * it / (ms * 1e-3),
                          "g": list(g.astuple()) if hasattr(g, "astuple") else (list(g) if g else None)}
