@@ -155,3 +155,34 @@ def test_dist_schedule_matches_layout(rg):
     pl = rg.dist.schedule("srad", 8192, 8192, 8, 0, 100, roi=(0, 127, 0, 127))
     assert (pl["top"], pl["bot"], pl["period"], pl["send_up"], pl["send_down"]) == (0, 16, 8, 0, 8)
     assert (pl["cone_r0"], pl["cone_r1"], pl["cone_c0"], pl["cone_c1"]) == (0, 330, 0, 330)
+
+
+def test_full_size_local_slabs_bitwise(rg):
+    # BASELINE configs[2] / [3] at full size through the row-slab path with P = 8 slabs on one GPU
+    # (LOCAL communicator: the same schedule, overlap split and halos as the NCCL path), in the
+    # granularity the bench tunes: bitwise equal to the single-GPU solve.
+    N, it = 16384, 1000
+    T, Pw = synth.hotspot_inputs(N, N)
+    c = rg.rodinia_hotspot_coeffs_rodinia(N, N, N * 31.25e-6, N * 31.25e-6)
+    g, _ = rg.rodinia_tune_pruned("hotspot", N // 8, N, it, keep=4, reps=1)
+    t, p = torch.from_numpy(T).cuda(), torch.from_numpy(Pw).cuda()
+    del T, Pw
+    ref = rg.rodinia_hotspot(t, p, it, coeffs=c, g=g)
+    comm = rg.dist.HaloComm.local_slabs(8)
+    ts, ps = _split(rg, t, 8), _split(rg, p, 8)
+    outs = [torch.empty_like(x) for x in ts]
+    comm.hotspot(ts, ps, outs, N, it, coeffs=c, g=g)
+    torch.cuda.synchronize()
+    assert torch.equal(torch.cat(outs), ref), g.astuple()
+    del ts, ps, outs, ref, t, p
+    M, n = 8192, 100
+    J = synth.srad_input(M, M)
+    for g in [(4, 1, 1, 3, 8, 1, rg.RODINIA_STREAM), None]:
+        ref = torch.from_numpy(J).cuda()
+        g1 = None if g is None else g[:4] + (1,) + g[5:]
+        rg.rodinia_srad(ref, 0, 127, 0, 127, 0.5, n, g=g1 if g is not None else (4, 1, 1, 2, 1, 1, rg.RODINIA_STREAM))
+        js = _split(rg, torch.from_numpy(J).cuda(), 8)
+        comm.srad(js, M, 0, 127, 0, 127, 0.5, n, g=g)
+        torch.cuda.synchronize()
+        assert torch.equal(torch.cat(js), ref), g
+    comm.close()
