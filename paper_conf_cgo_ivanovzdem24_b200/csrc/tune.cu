@@ -193,11 +193,39 @@ static void hotspot_stage1(std::vector<rodinia_granularity>* out) {
     }
 }
 
-static void hotspot_stage2(const rodinia_granularity& base, std::vector<rodinia_granularity>* out) {
+// Stage 2: block factors of one instantiation.  For the stream family the chunk height also gets
+// "wave-fitted" candidates: with S resident CTAs per wave (occupancy x SMs) and B bands, chunks
+// such that B x chunks fills w whole waves (w = 1..4, 8, 9) -- the fixed list alone leaves a
+// partial last wave on slab shapes (2048-row slabs at 8 ranks: 2.2 waves at by = 6).
+static void hotspot_stage2(const rodinia_granularity& base, int64_t R, int64_t C, std::vector<rodinia_granularity>* out) {
     rodinia_granularity g = base;
     if (g.flags & RODINIA_STREAM) {
+        std::vector<int> bys = {2, 3, 4, 6, 8, 12, 16, 24};
+        const int n = hotspot::num_variants();
+        int slots = 0;
+        for (int i = 0; i < n; ++i) {
+            rodinia_granularity vg;
+            const void* fn;
+            const char* key;
+            int threads;
+            hotspot::variant_info(i, &vg, &fn, &key, &threads);
+            if (vg.thread_x == g.thread_x && vg.temporal == g.temporal && vg.flags == g.flags) {
+                DeviceInfo di;
+                if (device_info(&di) == RODINIA_OK) slots = ctas_per_sm(fn, threads, 0) * di.sms;
+                break;
+            }
+        }
+        const int ow = 32 * g.thread_x - 2 * g.temporal;
+        const int64_t bands = ow > 0 ? (C + ow - 1) / ow : 0;
+        if (slots > 0 && bands > 0 && bands <= slots) {
+            for (int w : {1, 2, 3, 4, 8, 9}) {
+                const int64_t chunks = (int64_t)w * (slots / bands);
+                const int64_t by = (R + 16 * chunks - 1) / (16 * chunks);
+                if (by >= 1 && by <= 256 && std::find(bys.begin(), bys.end(), (int)by) == bys.end()) bys.push_back((int)by);
+            }
+        }
         for (int bx : {1, 2})
-            for (int by : {2, 3, 4, 6, 8, 12, 16, 24}) { g.block_x = bx; g.block_y = by; out->push_back(g); }
+            for (int by : bys) { g.block_x = bx; g.block_y = by; out->push_back(g); }
     } else {
         static const int bxy[][2] = {{1, 1}, {2, 1}, {3, 1}, {4, 1}, {7, 1}, {1, 2}, {2, 2}, {4, 4}};
         for (auto& b : bxy) { g.block_x = b[0]; g.block_y = b[1]; out->push_back(g); }
@@ -318,7 +346,7 @@ static rodinia_status tune_hotspot(const rodinia_problem& p, int reps, rodinia_g
     }
     for (auto& t : tops) {
         std::vector<rodinia_granularity> stage2;
-        hotspot_stage2(t, &stage2);
+        hotspot_stage2(t, R, C, &stage2);
         for (auto& g : stage2) {
             bool seen = false;
             for (auto& r : *rows) seen = seen || (memcmp(&r.g, &g, sizeof g) == 0);
