@@ -368,6 +368,7 @@ __global__ void __launch_bounds__(32, OCC)
     constexpr int SW = 32 * V;
     constexpr int OW = SW - 2 * H;
     static_assert(OW > 0, "band narrower than its halo");
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // launched as a programmatic dependent
     const int sc0 = (int)threadIdx.x * V;
     const int y0 = blockIdx.y * chunk;
     const int y1 = min(y0 + chunk, R);
@@ -510,7 +511,18 @@ static void launch_stream(const StreamVariant* sv, int bx, int by, const float* 
     const int vec_ok = (C % sv->v == 0) && (sv->h % sv->v == 0) &&
                        ((reinterpret_cast<uintptr_t>(tin) | reinterpret_cast<uintptr_t>(p) |
                          reinterpret_cast<uintptr_t>(tout)) % (4 * sv->v) == 0);
-    sv->fn<<<grid, 32, 0, s>>>(tin, p, tout, R, C, chunk, bx, cf, vec_ok);
+    // programmatic dependent of the preceding kernel (hs_stream waits with griddepcontrol.wait
+    // before touching memory): the launch of step-block k+1 overlaps the drain of step-block k
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(32);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, sv->fn, tin, p, tout, R, C, chunk, bx, cf, vec_ok);
     count_launch();
 }
 
