@@ -323,7 +323,8 @@ rodinia_status rodinia_comm_destroy(rodinia_comm* comm);
  * srad: D = granularity temporal (a NULL/zero granularity: min(8, rows per slab / 2)), halos D
  * above / 2D below (one iteration reads rows i-1..i+2), sends 2D up / D down.
  * r1..c2: the srad ROI (ignored for hotspot).  Errors: RODINIA_E_INVALID (arguments, other
- * kernels: pathfinder and lud are replicas only), RODINIA_E_ILLEGAL_FACTOR (slab thinner than the
+ * kernels: pathfinder is replicas only, lud has its own 2-D block-cyclic rodinia_lud_dist),
+ * RODINIA_E_ILLEGAL_FACTOR (slab thinner than the
  * halo), granularity errors as for the single-GPU call. */
 typedef struct {
     int64_t row0, own;
@@ -356,6 +357,28 @@ rodinia_status rodinia_srad_dist(rodinia_comm* comm, void* J_local, int64_t glob
                                  int64_t cols, int64_t r1, int64_t r2, int64_t c1, int64_t c2,
                                  float lambda, int32_t niter, const rodinia_granularity* g,
                                  void* stream);
+
+/* 2-D block-cyclic multi-GPU LU (the last step).  The same
+ * operation as rodinia_lud (Doolittle, no pivoting, packed in place; DESIGN.md §3 L1-L6) on a
+ * prow x pcol process grid, rank r = pr * pcol + pc, blocks of NB = 128: global block (I, J)
+ * (rows [128 I, 128 I + 128) x cols [128 J, ...), the last ones partial) lives on rank
+ * (I mod prow, J mod pcol).  a_local: this rank's local matrix (LOCAL communicator: an array of
+ * `nranks` local-matrix pointers, rank order), device, row-major, mloc x nloc with leading
+ * dimension nloc (rodinia_lud_dist_layout): the rank's block rows in increasing I by its block
+ * columns in increasing J.  Factored in place.  Per block column k: the owner of A_kk factors
+ * it and broadcasts it (ncclBroadcast; LOCAL: copies), process column k mod pcol solves
+ * L_Ik = A_Ik U_kk^-1, process row k mod prow solves U_kJ = L_kk^-1 A_kJ, the L panels travel
+ * along process rows and the U panels along process columns (ncclSend/ncclRecv, as hi/lo TF32
+ * operand images), and every rank applies A_IJ -= L_Ik U_kJ to its trailing blocks on the tensor
+ * cores (3xTF32, the panel-128 update).  Per element the arithmetic does not depend on the grid:
+ * every grid (1 x 1 included) gives the same bits.  Stream-ordered on `stream`; scratch is
+ * stream-ordered (cudaMallocAsync) and released at the end.  Errors: RODINIA_E_INVALID (grid
+ * != nranks, null pointers), RODINIA_E_NOMEM, RODINIA_E_NCCL, RODINIA_E_CUDA. */
+rodinia_status rodinia_lud_dist(rodinia_comm* comm, void* a_local, int64_t n, int32_t prow, int32_t pcol,
+                                void* stream);
+/* Host only: local matrix shape (rows mloc, columns nloc) of `rank` for rodinia_lud_dist. */
+rodinia_status rodinia_lud_dist_layout(int64_t n, int32_t prow, int32_t pcol, int32_t rank, int64_t* mloc,
+                                       int64_t* nloc);
 
 /* Split a *total* coarsening factor over `ndims` (1..3) dimensions (footnote 4,
  * "for a total factor of 16, we will coarsen the 3 dimensions with 4, 2, and 2

@@ -148,6 +148,8 @@ _SIGS = {
     "rodinia_comm_destroy": ([_vp], _i32),
     "rodinia_hotspot_dist": ([_vp, _vp, _vp, _vp, _i64, _i64, _i32, _PC, _PG, _vp], _i32),
     "rodinia_srad_dist": ([_vp, _vp, _i64, _i64, _i64, _i64, _i64, _i64, _f32, _i32, _PG, _vp], _i32),
+    "rodinia_lud_dist": ([_vp, _vp, _i64, _i32, _i32, _vp], _i32),
+    "rodinia_lud_dist_layout": ([_i64, _i32, _i32, _i32, ctypes.POINTER(_i64), ctypes.POINTER(_i64)], _i32),
     "rodinia_dist_schedule": ([_i32, _i64, _i64, _i32, _i32, _i32, _i64, _i64, _i64, _i64, _PG, _vp], _i32),
 }
 

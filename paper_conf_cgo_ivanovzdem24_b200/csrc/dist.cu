@@ -718,3 +718,194 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
     }
     return st;
 }
+
+// ===================================================================== 2-D block-cyclic LU
+// SURVEY §8(f) #3 ("then a 2-D block-cyclic multi-GPU LU"), DESIGN.md §6.  Process grid
+// prow x pcol (rank r = pr * pcol + pc), NB = 128 blocks; global block (I, J) lives on rank
+// (I mod prow, J mod pcol).  Local matrix: the rank's block rows in increasing I, its block
+// columns in increasing J, row-major, leading dimension = local columns (rodinia_lud_dist_layout).
+// Right-looking, per block column k (owner (pk, qk) = (k mod prow, k mod pcol)):
+//   1. (pk, qk) factors A_kk (ldist::diag) and broadcasts its images to every rank;
+//   2. process column qk solves its L_Ik, process row pk its U_kJ (ldist::trsm), each writing
+//      the hi/lo operand image of its panel;
+//   3. L images travel along process rows, U images along process columns (send/recv);
+//   4. every rank updates its trailing blocks (ldist::update, tensor cores).
+namespace rg {
+static int64_t bc_extent(int64_t n, int P, int p) {  // rows of the global blocks I = p (mod P)
+    const int64_t nb = (n + ldist::NB - 1) / ldist::NB;
+    int64_t e = 0;
+    for (int64_t I = p; I < nb; I += P) e += std::min<int64_t>(ldist::NB, n - I * ldist::NB);
+    return e;
+}
+static int64_t bc_blocks_le(int64_t k, int P, int p) {  // local blocks I = p (mod P) with I <= k
+    return k < p ? 0 : (k - p) / P + 1;
+}
+struct LudRank {
+    int r, pr, pc;
+    float* A;
+    int64_t mloc, nloc;
+    float** slot;
+    float* mimg;
+    float* ia;
+    float* ib;
+};
+}  // namespace rg
+
+extern "C" rodinia_status rodinia_lud_dist_layout(int64_t n, int32_t prow, int32_t pcol, int32_t rank,
+                                                  int64_t* mloc, int64_t* nloc) {
+    if (n < 1 || prow < 1 || pcol < 1 || rank < 0 || rank >= prow * pcol || !mloc || !nloc)
+        return set_error(RODINIA_E_INVALID, "lud_dist_layout: bad arguments");
+    *mloc = bc_extent(n, prow, rank / pcol);
+    *nloc = bc_extent(n, pcol, rank % pcol);
+    return RODINIA_OK;
+}
+
+extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64_t n, int32_t prow, int32_t pcol,
+                                           void* stream) {
+    if (!c || !a_local || n < 1 || prow < 1 || pcol < 1)
+        return set_error(RODINIA_E_INVALID, "lud_dist: bad arguments");
+    if (prow * pcol != c->nranks)
+        return set_error(RODINIA_E_INVALID, "lud_dist: process grid %d x %d != %d ranks", prow, pcol, c->nranks);
+    if (n > (int64_t)1 << 20) return set_error(RODINIA_E_INVALID, "lud_dist: n too large");
+    std::lock_guard<std::mutex> lk(c->mu);
+    cudaStream_t s = (cudaStream_t)stream;
+    const int P = c->nranks;
+    std::vector<LudRank> rk;
+    for (int r = 0; r < P; ++r) {
+        if (c->kind != 1 && r != c->rank) continue;
+        LudRank x;
+        memset(&x, 0, sizeof x);
+        x.r = r;
+        x.pr = r / pcol;
+        x.pc = r % pcol;
+        x.A = (float*)arg_ptr(c, a_local, rk.size());
+        x.mloc = bc_extent(n, prow, x.pr);
+        x.nloc = bc_extent(n, pcol, x.pc);
+        rk.push_back(x);
+    }
+    auto cleanup = [&]() {
+        for (auto& x : rk)
+            for (void* p : {(void*)x.slot, (void*)x.mimg, (void*)x.ia, (void*)x.ib})
+                if (p) cudaFreeAsync(p, s);
+    };
+    for (auto& x : rk) {
+        if ((x.mloc > 0 && x.nloc > 0 && !x.A) ||
+            cudaMallocAsync((void**)&x.slot, sizeof(float*), s) != cudaSuccess ||
+            cudaMallocAsync((void**)&x.mimg, ldist::mimg_floats() * sizeof(float), s) != cudaSuccess ||
+            cudaMallocAsync((void**)&x.ia, ldist::img_floats(std::max<int64_t>(x.mloc, 1)) * sizeof(float), s) !=
+                cudaSuccess ||
+            cudaMallocAsync((void**)&x.ib, ldist::img_floats(std::max<int64_t>(x.nloc, 1)) * sizeof(float), s) !=
+                cudaSuccess) {
+            cudaGetLastError();
+            cleanup();
+            return set_error(RODINIA_E_NOMEM, "lud_dist: scratch allocation failed");
+        }
+        rodinia_status st = ldist::set_slot(x.slot, x.A, s);
+        if (st != RODINIA_OK) { cleanup(); return st; }
+    }
+    NcclApi* api = nullptr;
+    if (c->kind != 1 && P > 1) {
+        rodinia_status st = nccl_api(&api);
+        if (st != RODINIA_OK) { cleanup(); return st; }
+    }
+    const int64_t NB = ldist::NB, nb = (n + NB - 1) / NB;
+    rodinia_status st = RODINIA_OK;
+    auto find = [&](int r) -> LudRank* {
+        for (auto& x : rk)
+            if (x.r == r) return &x;
+        return nullptr;
+    };
+#define LD_TRY(x)                        \
+    do {                                 \
+        st = (x);                        \
+        if (st != RODINIA_OK) goto done; \
+    } while (0)
+    for (int64_t k = 0; k < nb; ++k) {
+        const int pk = (int)(k % prow), qk = (int)(k % pcol), root = pk * pcol + qk;
+        const int bk = (int)std::min<int64_t>(NB, n - k * NB);
+        const int64_t lrk = (k / prow) * NB, lck = (k / pcol) * NB;  // block (k, k) on its owner
+        if (LudRank* o = find(root)) LD_TRY(ldist::diag(o->A + lrk * o->nloc + lck, (int)o->nloc, bk, o->mimg, s));
+        if (k == nb - 1) break;
+        // 1. the diagonal block's images to every rank
+        if (P > 1) {
+            const size_t cnt = ldist::mimg_floats();
+            if (c->kind == 1) {
+                LudRank* o = find(root);
+                for (auto& x : rk)
+                    if (x.r != root)
+                        if (cudaMemcpyAsync(x.mimg, o->mimg, cnt * sizeof(float), cudaMemcpyDeviceToDevice, s) !=
+                            cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist bcast", __FILE__, __LINE__); goto done; }
+            } else {
+                ncclResult_t e = api->Bcast(rk[0].mimg, rk[0].mimg, cnt, ncclFloat32, root, c->nccl, s);
+                if (e != ncclSuccess) { st = set_error(RODINIA_E_NCCL, "lud_dist bcast: %s", api->GetErrorString(e)); goto done; }
+            }
+        }
+        // 2. panel solves: L_Ik on process column qk, U_kJ on process row pk
+        for (auto& x : rk) {
+            const int64_t lr0 = bc_blocks_le(k, prow, x.pr) * NB, lc0 = bc_blocks_le(k, pcol, x.pc) * NB;
+            if (x.pc == qk && x.mloc > lr0)
+                LD_TRY(ldist::trsm(x.A + lr0 * x.nloc + lck, (int)x.nloc, true, (int)(x.mloc - lr0), x.ia,
+                                   ldist::img_groups(x.mloc - lr0), x.mimg, s));
+            if (x.pr == pk && x.nloc > lc0)
+                LD_TRY(ldist::trsm(x.A + lrk * x.nloc + lc0, (int)x.nloc, false, (int)(x.nloc - lc0), x.ib,
+                                   ldist::img_groups(x.nloc - lc0), x.mimg, s));
+        }
+        // 3. L images along process rows (from (pr, qk)), U images along process columns (from (pk, pc))
+        if (P > 1) {
+            if (c->kind == 1) {
+                for (auto& x : rk) {
+                    const int64_t rows = x.mloc - bc_blocks_le(k, prow, x.pr) * NB;
+                    const int64_t cols = x.nloc - bc_blocks_le(k, pcol, x.pc) * NB;
+                    if (x.pc != qk && rows > 0) {
+                        LudRank* src = find(x.pr * pcol + qk);
+                        if (cudaMemcpyAsync(x.ia, src->ia, ldist::img_floats(rows) * sizeof(float),
+                                            cudaMemcpyDeviceToDevice, s) != cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist L image", __FILE__, __LINE__); goto done; }
+                    }
+                    if (x.pr != pk && cols > 0) {
+                        LudRank* src = find(pk * pcol + x.pc);
+                        if (cudaMemcpyAsync(x.ib, src->ib, ldist::img_floats(cols) * sizeof(float),
+                                            cudaMemcpyDeviceToDevice, s) != cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist U image", __FILE__, __LINE__); goto done; }
+                    }
+                }
+            } else {
+                LudRank& x = rk[0];
+                const int64_t rows = x.mloc - bc_blocks_le(k, prow, x.pr) * NB;
+                const int64_t cols = x.nloc - bc_blocks_le(k, pcol, x.pc) * NB;
+                ncclResult_t e = api->GroupStart();
+                if (rows > 0 && pcol > 1) {
+                    const size_t cnt = ldist::img_floats(rows);
+                    if (x.pc == qk) {
+                        for (int q = 0; q < pcol && e == ncclSuccess; ++q)
+                            if (q != qk) e = api->Send(x.ia, cnt, ncclFloat32, x.pr * pcol + q, c->nccl, s);
+                    } else if (e == ncclSuccess) {
+                        e = api->Recv(x.ia, cnt, ncclFloat32, x.pr * pcol + qk, c->nccl, s);
+                    }
+                }
+                if (cols > 0 && prow > 1 && e == ncclSuccess) {
+                    const size_t cnt = ldist::img_floats(cols);
+                    if (x.pr == pk) {
+                        for (int p = 0; p < prow && e == ncclSuccess; ++p)
+                            if (p != pk) e = api->Send(x.ib, cnt, ncclFloat32, p * pcol + x.pc, c->nccl, s);
+                    } else {
+                        e = api->Recv(x.ib, cnt, ncclFloat32, pk * pcol + x.pc, c->nccl, s);
+                    }
+                }
+                ncclResult_t e2 = api->GroupEnd();
+                if (e == ncclSuccess) e = e2;
+                if (e != ncclSuccess) { st = set_error(RODINIA_E_NCCL, "lud_dist panels: %s", api->GetErrorString(e)); goto done; }
+            }
+        }
+        // 4. local trailing updates
+        for (auto& x : rk) {
+            const int64_t lr0 = bc_blocks_le(k, prow, x.pr) * NB, lc0 = bc_blocks_le(k, pcol, x.pc) * NB;
+            const int64_t rows = x.mloc - lr0, cols = x.nloc - lc0;
+            if (rows > 0 && cols > 0)
+                LD_TRY(ldist::update(x.slot, (int)x.nloc, (int)lr0, (int)rows, (int)lc0, (int)cols, x.ia,
+                                     ldist::img_groups(rows), x.ib, ldist::img_groups(cols), s));
+        }
+    }
+done:
+#undef LD_TRY
+    cleanup();
+    return st;
+}

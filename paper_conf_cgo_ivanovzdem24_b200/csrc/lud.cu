@@ -29,6 +29,7 @@
 
 #include "rg_internal.h"
 #include "lud_tc.cuh"
+#include "workloads.h"
 
 namespace rg {
 
@@ -813,6 +814,440 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
     if (st == RODINIA_OK) tune_cache_store(RODINIA_LUD, pr, *best, best_ms);
     return st;
 }
+
+// ================================================================== 2-D block-cyclic distributed LU
+// SURVEY §8(f) #3 (the last step: "then a 2-D block-cyclic multi-GPU LU"), DESIGN.md §6.
+// Building blocks of rodinia_lud_dist (dist.cu), each acting on one rank's local matrix
+// (row-major, leading dimension lda) in NB = 128 blocks:
+//   ldist::diag    factor the diagonal block A_kk = L_kk U_kk in place (lud_diag128, one CTA)
+//                  and write the images the solves read (U_kk row-major, L_kk transposed,
+//                  RN(1/u_jj)), the payload broadcast from the block's owner;
+//   ldist::trsm    L_Ik = A_Ik U_kk^-1 (local rows) or U_kJ = L_kk^-1 A_kJ (local columns)
+//                  in place, one thread per row / column (lud_trsm128), writing the hi/lo
+//                  TF32 operand image of the update as it goes (the payload sent along the
+//                  process row / column);
+//   ldist::update  the local trailing update A_IJ -= L_Ik U_kJ on the tensor cores
+//                  (lud_tc_update2, 3xTF32, the single-GPU panel-128 update kernel).
+// Per element the operations and their order depend only on the global element, never on
+// the process grid, so every grid gives the same bits (tests/test_gpu_lud_dist.py).
+// Doolittle's sequence (reading L5): subtractions in ascending k, L divided by its pivot after
+// its k < j terms; products fused (FMA); quotients = IEEE quotients formed from the pivot's
+// correctly rounded reciprocal (div_rcp).
+constexpr int LD_NB = 128;
+constexpr int D128_LD = 132;                   // 16-byte aligned rows, conflict-free row reads
+constexpr int D128_IMG = 128 * D128_LD;        // one 128 x 128 image padded to D128_LD
+constexpr size_t d128_mimg_floats() { return (size_t)2 * D128_IMG + 128; }
+
+// RN(a / b) from rb = RN(1 / b) (Markstein): q0 = RN(a rb) lies within one ulp of a/b, the
+// residual a - q0 b is exact in one FMA, and RN(q0 + residual * rb) is the correctly rounded
+// quotient in the absence of underflow/overflow -- the value __fdiv_rn returns, with the
+// reciprocal computed once per pivot.  (b = 0 gives NaN where __fdiv_rn gives inf; zero pivots
+// are outside the method, reading L1.)
+__device__ __forceinline__ float div_rcp(float a, float b, float rb) {
+    const float q0 = __fmul_rn(a, rb);
+    const float e = __fmaf_rn(-q0, b, a);
+    return __fmaf_rn(e, rb, q0);
+}
+
+// Right-looking LU of the rs x rs leading part of a 32 x 32 block held one row per lane
+// (a[j] = element (lane, j)), one warp.  Step kk: lane kk publishes its final row through the
+// shared-memory buffer rowbuf (double-buffered, broadcast reads), lanes kk < i < rs form
+// l_ik = a_ik / u_kk and subtract l_ik u_kj for j > kk (others use l = 0: row unchanged).
+// rinv[i] = RN(1/u_ii) for i < rs.
+__device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rowbuf, float* rinv) {
+    float myrb = 0.f;
+#pragma unroll
+    for (int kk = 0; kk < 32; ++kk) {
+        if (kk >= rs) break;  // uniform
+        float* row = rowbuf + 32 * (kk & 1);
+        if (lane == kk) {
+#pragma unroll
+            for (int q = kk / 4; q < 8; ++q)
+                *reinterpret_cast<float4*>(row + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
+        }
+        __syncwarp();
+        float u[32];
+#pragma unroll
+        for (int q = kk / 4; q < 8; ++q) {
+            const float4 t = *reinterpret_cast<const float4*>(row + 4 * q);
+            u[4 * q] = t.x; u[4 * q + 1] = t.y; u[4 * q + 2] = t.z; u[4 * q + 3] = t.w;
+        }
+        const float rb = __frcp_rn(u[kk]);
+        if (lane == kk) myrb = rb;
+        const bool below = lane > kk && lane < rs;
+        const float l = below ? div_rcp(a[kk], u[kk], rb) : 0.f;
+        a[kk] = below ? l : a[kk];
+#pragma unroll
+        for (int j = kk + 1; j < 32; ++j) a[j] = __fmaf_rn(-l, u[j], a[j]);
+    }
+    if (lane < rs) rinv[lane] = myrb;
+}
+
+// One CTA of 256 threads factors the r x r block at A (r <= 128, row stride lda) in shared
+// memory (rows/columns >= r are zeros and stay zeros), right-looking over 32-wide sub-panels:
+// threads 0..95 solve a sub-panel's L rows below the factored diagonal sub-block, threads
+// 128..223 its U columns right of it; then warp 0 applies the rank-32 update to the NEXT
+// diagonal sub-block and factors it (diag32_factor) while warps 1..7 update the rest of the
+// trailing block (4 x 4 register tiles).  Outputs: the block in A, and mimg = [U image |
+// L^T image | RN(1/u_jj)] (d128_mimg_floats), written with bulk copies.
+__global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int lda, int r, float* __restrict__ mimg) {
+    constexpr int LD = D128_LD;
+    extern __shared__ __align__(128) float S[];  // 132 x LD, then the transposed image 128 x LD
+    __shared__ __align__(16) float rowbuf[64];
+    __shared__ __align__(16) float rinv[128];
+    __shared__ __align__(8) uint64_t mbar;
+    float* T = S + 132 * LD;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const bool bulk = r == 128 && (lda & 3) == 0 && ((uintptr_t)A & 15) == 0;
+    if (bulk) {  // 128 row copies of 512 B
+        if (tid == 0) {
+            tc::mbar_init(&mbar, 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            tc::mbar_expect_tx(&mbar, 128 * 512);
+        }
+        __syncthreads();
+        if (tid < 128) tc::bulk_g2s(S + tid * LD, A + (size_t)tid * lda, 512, &mbar);
+    } else {
+        float v[64];
+#pragma unroll
+        for (int q = 0; q < 64; ++q) {
+            const int e = tid + 256 * q, i = e >> 7, j = e & 127;
+            v[q] = (i < r && j < r) ? A[(size_t)i * lda + j] : 0.f;
+        }
+#pragma unroll
+        for (int q = 0; q < 64; ++q) {
+            const int e = tid + 256 * q, i = e >> 7, j = e & 127;
+            S[i * LD + j] = v[q];
+        }
+    }
+    for (int e = tid; e < 4 * LD + 128 * 4; e += 256) {  // zero padding: rows 128..131, cols 128..131
+        if (e < 4 * LD) S[128 * LD + e] = 0.f;
+        else S[((e - 4 * LD) >> 2) * LD + 128 + ((e - 4 * LD) & 3)] = 0.f;
+    }
+    if (bulk) tc::mbar_wait(&mbar, 0);
+    __syncthreads();
+    if (warp == 0) {  // the first diagonal sub-block
+        float a[32];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const float4 t = *reinterpret_cast<const float4*>(S + lane * LD + 4 * q);
+            a[4 * q] = t.x; a[4 * q + 1] = t.y; a[4 * q + 2] = t.z; a[4 * q + 3] = t.w;
+        }
+        diag32_factor(a, min(32, r), lane, rowbuf, rinv);
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+            *reinterpret_cast<float4*>(S + lane * LD + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
+    }
+    __syncthreads();
+#pragma unroll 1
+    for (int p = 0; p + 32 < r; p += 32) {
+        const int rest = r - p - 32;  // rows below / columns right of the factored sub-block
+        if (tid < rest) {
+            // L row i: x_j = (a_ij - sum_{k<j} x_k u_kj) / u_jj over the sub-block's columns
+            float* xr = S + (p + 32 + tid) * LD + p;
+            float x[32];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float4 t = *reinterpret_cast<const float4*>(xr + 4 * q);
+                x[4 * q] = t.x; x[4 * q + 1] = t.y; x[4 * q + 2] = t.z; x[4 * q + 3] = t.w;
+            }
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+                const float* ur = S + (p + j) * LD + p;
+                float u[32];
+#pragma unroll
+                for (int q = j / 4; q < 8; ++q) {
+                    const float4 t = *reinterpret_cast<const float4*>(ur + 4 * q);
+                    u[4 * q] = t.x; u[4 * q + 1] = t.y; u[4 * q + 2] = t.z; u[4 * q + 3] = t.w;
+                }
+                x[j] = div_rcp(x[j], u[j], rinv[p + j]);
+#pragma unroll
+                for (int j2 = j + 1; j2 < 32; ++j2) x[j2] = __fmaf_rn(-x[j], u[j2], x[j2]);
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                *reinterpret_cast<float4*>(xr + 4 * q) = make_float4(x[4 * q], x[4 * q + 1], x[4 * q + 2], x[4 * q + 3]);
+        } else if (tid >= 128 && tid - 128 < rest) {
+            // U column c: y_i = a_ic - sum_{k<i} l_ik y_k (unit-lower sub-block)
+            const int c = p + 32 + (tid - 128);
+            float y[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i) y[i] = S[(p + i) * LD + c];
+#pragma unroll
+            for (int k = 0; k < 32; ++k)
+#pragma unroll
+                for (int i = k + 1; i < 32; ++i) y[i] = __fmaf_rn(-S[(p + i) * LD + p + k], y[k], y[i]);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) S[(p + i) * LD + c] = y[i];
+        }
+        __syncthreads();
+        const int nb = p + 32;
+        if (warp == 0) {
+            // the next diagonal sub-block: its rank-32 update, then its factorisation
+            float lr[32], a[32];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float4 t = *reinterpret_cast<const float4*>(S + (nb + lane) * LD + p + 4 * q);
+                lr[4 * q] = -t.x; lr[4 * q + 1] = -t.y; lr[4 * q + 2] = -t.z; lr[4 * q + 3] = -t.w;
+                const float4 c = *reinterpret_cast<const float4*>(S + (nb + lane) * LD + nb + 4 * q);
+                a[4 * q] = c.x; a[4 * q + 1] = c.y; a[4 * q + 2] = c.z; a[4 * q + 3] = c.w;
+            }
+#pragma unroll
+            for (int k = 0; k < 32; ++k) {
+                const float4* ur = reinterpret_cast<const float4*>(S + (p + k) * LD + nb);
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    const float4 u = ur[q];
+                    a[4 * q] = __fmaf_rn(lr[k], u.x, a[4 * q]);
+                    a[4 * q + 1] = __fmaf_rn(lr[k], u.y, a[4 * q + 1]);
+                    a[4 * q + 2] = __fmaf_rn(lr[k], u.z, a[4 * q + 2]);
+                    a[4 * q + 3] = __fmaf_rn(lr[k], u.w, a[4 * q + 3]);
+                }
+            }
+            diag32_factor(a, min(32, rest), lane, rowbuf, rinv + nb);
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                *reinterpret_cast<float4*>(S + (nb + lane) * LD + nb + 4 * q) =
+                    make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
+        } else {
+            // rank-32 update of the rest of [nb, r)^2 (tiles may reach into the zero padding)
+            const int nt = (rest + 3) / 4;
+            for (int t = tid - 32; t < nt * nt; t += 224) {
+                const int ti = t / nt, tj = t - (t / nt) * nt;
+                if (ti < 8 && tj < 8) continue;  // the next diagonal sub-block (warp 0)
+                const int i0 = nb + 4 * ti, j0 = nb + 4 * tj;
+                float acc[4][4];
+#pragma unroll
+                for (int a = 0; a < 4; ++a) {
+                    const float4 v = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0);
+                    acc[a][0] = v.x; acc[a][1] = v.y; acc[a][2] = v.z; acc[a][3] = v.w;
+                }
+#pragma unroll 8
+                for (int k = 0; k < 32; ++k) {
+                    const float4 u = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
+#pragma unroll
+                    for (int a = 0; a < 4; ++a) {
+                        const float l = -S[(i0 + a) * LD + p + k];
+                        acc[a][0] = __fmaf_rn(l, u.x, acc[a][0]);
+                        acc[a][1] = __fmaf_rn(l, u.y, acc[a][1]);
+                        acc[a][2] = __fmaf_rn(l, u.z, acc[a][2]);
+                        acc[a][3] = __fmaf_rn(l, u.w, acc[a][3]);
+                    }
+                }
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0) =
+                        make_float4(acc[a][0], acc[a][1], acc[a][2], acc[a][3]);
+            }
+        }
+        __syncthreads();
+    }
+    // outputs: the transposed image in shared memory, then bulk stores (A rows, images, 1/u)
+    for (int e = tid; e < 128 * 128; e += 256) {
+        const int i = e >> 7, k = e & 127;
+        T[k * LD + i] = S[i * LD + k];
+    }
+    for (int e = tid; e < 128 * 4; e += 256) T[(e >> 2) * LD + 128 + (e & 3)] = 0.f;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    if (tid == 0) {
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg),
+                     "r"(tc::smem_u32(S)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + D128_IMG),
+                     "r"(tc::smem_u32(T)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + 2 * D128_IMG),
+                     "r"(tc::smem_u32(rinv)), "r"(512u) : "memory");
+    }
+    if (bulk) {
+        if (tid < 128)
+            asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], 512;" ::"l"(A + (size_t)tid * lda),
+                         "r"(tc::smem_u32(S + tid * LD)) : "memory");
+    } else {
+        for (int e = tid; e < r * 128; e += 256) {
+            const int i = e >> 7, j = e & 127;
+            if (j < r) A[(size_t)i * lda + j] = S[i * LD + j];
+        }
+    }
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+constexpr size_t d128_smem() { return (size_t)(132 + 128) * D128_LD * sizeof(float); }
+
+// Triangular solves against the factored 128 x 128 diagonal block (mimg from lud_diag128),
+// 64 threads per CTA, one thread per row (lower: L = A U^-1, row t at A + t*lda) or per
+// column (upper: U = L^-1 A, column t at A + t, rows at stride lda), `count` of them.  Both are
+// the substitution x_j -= sum_{k<j} x_k M[k][j] with M (U, or L transposed) bulk-copied into
+// shared memory, in four 32-wide pieces: the solved values of earlier pieces (kept per thread
+// in shared memory) are applied first (left-looking, 16 independent FFMA2 chains), then the
+// 32-step substitution inside the piece (lower: divided by the pivot after its k < j terms).
+// Each solved piece is written to A and, split hi/lo, to the tensor-core operand image `img`
+// (ng 8-row groups) of the update, image row = thread index.
+constexpr int TR_T = 64, TR_RLD = 129;
+constexpr size_t trsm_smem() { return ((size_t)D128_IMG + 128 + (size_t)TR_T * TR_RLD) * sizeof(float); }
+
+__device__ __forceinline__ void trsm_load(const float* A, int lda, bool lower, bool vec, bool own, int idx, int c0,
+                                          float2 (&x)[16]) {
+    if (!own) {
+#pragma unroll
+        for (int q = 0; q < 16; ++q) x[q] = make_float2(0.f, 0.f);
+    } else if (lower && vec) {
+        const float4* src = reinterpret_cast<const float4*>(A + (size_t)idx * lda + c0);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const float4 t = src[q];
+            x[2 * q] = make_float2(t.x, t.y);
+            x[2 * q + 1] = make_float2(t.z, t.w);
+        }
+    } else if (lower) {
+#pragma unroll
+        for (int q = 0; q < 16; ++q)
+            x[q] = make_float2(A[(size_t)idx * lda + c0 + 2 * q], A[(size_t)idx * lda + c0 + 2 * q + 1]);
+    } else {
+#pragma unroll
+        for (int q = 0; q < 16; ++q)
+            x[q] = make_float2(A[(size_t)(c0 + 2 * q) * lda + idx], A[(size_t)(c0 + 2 * q + 1) * lda + idx]);
+    }
+}
+
+__global__ void __launch_bounds__(TR_T) lud_trsm128(float* __restrict__ A, int lda, int lower_, int count,
+                                                   float* __restrict__ img, int ng, const float* __restrict__ mimg) {
+    constexpr int LD = D128_LD;
+    extern __shared__ __align__(128) float sm[];
+    __shared__ __align__(8) uint64_t mbar;
+    float* M = sm;
+    float* rinv = sm + D128_IMG;
+    float* R = rinv + 128;
+    const bool lower = lower_ != 0;
+    const int tid = threadIdx.x, idx = blockIdx.x * TR_T + tid;
+    const bool own = idx < count;
+    const bool vec = (lda & 3) == 0 && ((uintptr_t)A & 15) == 0;
+    if (tid == 0) {  // M and the pivots' reciprocals: two bulk copies
+        tc::mbar_init(&mbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        tc::mbar_expect_tx(&mbar, D128_IMG * 4 + 512);
+        tc::bulk_g2s(M, mimg + (lower ? 0 : D128_IMG), D128_IMG * 4, &mbar);
+        tc::bulk_g2s(rinv, mimg + 2 * D128_IMG, 512, &mbar);
+    }
+    float2 x[16], xn[16];
+    trsm_load(A, lda, lower, vec, own, idx, 0, x);
+    __syncthreads();
+    tc::mbar_wait(&mbar, 0);
+    float* Rt = R + tid * TR_RLD;
+#pragma unroll 1
+    for (int p = 0; p < 128; p += 32) {
+        if (p + 32 < 128) trsm_load(A, lda, lower, vec, own, idx, p + 32, xn);
+#pragma unroll 4
+        for (int k = 0; k < p; ++k) {
+            const float nl = -Rt[k];
+            const float2 nl2 = make_float2(nl, nl);
+            const float4* mr = reinterpret_cast<const float4*>(M + k * LD + p);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float4 m = mr[q];
+                x[2 * q] = __ffma2_rn(nl2, make_float2(m.x, m.y), x[2 * q]);
+                x[2 * q + 1] = __ffma2_rn(nl2, make_float2(m.z, m.w), x[2 * q + 1]);
+            }
+        }
+        float xs[32];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) { xs[2 * q] = x[q].x; xs[2 * q + 1] = x[q].y; }
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+            const float4* mr = reinterpret_cast<const float4*>(M + (p + j) * LD + p);
+            float mv[32];
+#pragma unroll
+            for (int q = j / 4; q < 8; ++q) {
+                const float4 m = mr[q];
+                mv[4 * q] = m.x; mv[4 * q + 1] = m.y; mv[4 * q + 2] = m.z; mv[4 * q + 3] = m.w;
+            }
+            if (lower) xs[j] = div_rcp(xs[j], mv[j], rinv[p + j]);
+#pragma unroll
+            for (int j2 = j + 1; j2 < 32; ++j2) xs[j2] = __fmaf_rn(-xs[j], mv[j2], xs[j2]);
+        }
+#pragma unroll
+        for (int j = 0; j < 32; ++j) Rt[p + j] = xs[j];
+        if (own) {
+            if (lower && vec) {
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                    *reinterpret_cast<float4*>(A + (size_t)idx * lda + p + 4 * q) =
+                        make_float4(xs[4 * q], xs[4 * q + 1], xs[4 * q + 2], xs[4 * q + 3]);
+            } else if (lower) {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) A[(size_t)idx * lda + p + j] = xs[j];
+            } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) A[(size_t)(p + j) * lda + idx] = xs[j];
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const float f[4] = {xs[4 * q], xs[4 * q + 1], xs[4 * q + 2], xs[4 * q + 3]};
+                tc::img_store4(img, ng, idx, p + 4 * q, f);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < 16; ++q) x[q] = xn[q];
+    }
+}
+
+namespace ldist {
+size_t mimg_floats() { return d128_mimg_floats(); }
+int img_groups(int64_t rows) { return (int)(((rows + 127) / 128 + 1) * 16); }
+size_t img_floats(int64_t rows) { return (size_t)16 * img_groups(rows) * tc::KC2 * 8; }
+
+rodinia_status diag(float* A, int lda, int r, float* mimg, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        RG_CUDA(cudaFuncSetAttribute((const void*)lud_diag128, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)d128_smem()));
+        attr = true;
+    }
+    lud_diag128<<<1, 256, d128_smem(), s>>>(A, lda, r, mimg);
+    RG_CUDA(cudaGetLastError());
+    count_launch();
+    return RODINIA_OK;
+}
+
+rodinia_status trsm(float* A, int lda, bool lower, int count, float* img, int ng, const float* mimg, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        RG_CUDA(cudaFuncSetAttribute((const void*)lud_trsm128, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)trsm_smem()));
+        attr = true;
+    }
+    if (count <= 0) return RODINIA_OK;
+    lud_trsm128<<<(count + TR_T - 1) / TR_T, TR_T, trsm_smem(), s>>>(A, lda, lower ? 1 : 0, count, img, ng, mimg);
+    RG_CUDA(cudaGetLastError());
+    count_launch();
+    return RODINIA_OK;
+}
+
+rodinia_status set_slot(float** slot, float* a, cudaStream_t s) {
+    lud_set_slot<<<1, 1, 0, s>>>(slot, a);
+    RG_CUDA(cudaGetLastError());
+    return RODINIA_OK;
+}
+
+rodinia_status update(float* const* slot, int lda, int r0, int m, int c0, int nn, const float* ia, int nga,
+                      const float* ib, int ngb, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update2, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)tc::smem_bytes2()));
+        attr = true;
+    }
+    if (m <= 0 || nn <= 0) return RODINIA_OK;
+    tc::Args a;
+    a.nrect = 1;
+    a.rect[0] = tc::make_rect(r0, c0, m, nn, 0, LD_NB);
+    a.rect[1] = a.rect[0];
+    const tc::Img im{ia, ib, r0, c0, nga, ngb, 0};
+    tc::lud_tc_update2<<<a.rect[0].tiles, 128, tc::smem_bytes2(), s>>>(slot, lda, a, im, -1);
+    RG_CUDA(cudaGetLastError());
+    count_launch();
+    return RODINIA_OK;
+}
+}  // namespace ldist
 
 }  // namespace rg
 

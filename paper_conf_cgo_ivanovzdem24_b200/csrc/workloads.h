@@ -71,4 +71,18 @@ float* engine_steps(Engine* e, float* cur, float* other, int i0, int i1, bool st
 rodinia_status take_sticky();
 }  // namespace srad
 
+// 2-D block-cyclic distributed LU building blocks (lud.cu; orchestrated by rodinia_lud_dist)
+namespace ldist {
+constexpr int NB = 128;                      // block size (the tensor-core update tile)
+size_t mimg_floats();                        // diagonal-block payload (U, L^T images, 1/u)
+int img_groups(int64_t rows);                // 8-row groups of an operand image for `rows`
+size_t img_floats(int64_t rows);             // floats of such an image (hi + lo, K = 128)
+rodinia_status diag(float* A, int lda, int r, float* mimg, cudaStream_t s);
+rodinia_status trsm(float* A, int lda, bool lower, int count, float* img, int ng, const float* mimg,
+                    cudaStream_t s);
+rodinia_status set_slot(float** slot, float* a, cudaStream_t s);
+rodinia_status update(float* const* slot, int lda, int r0, int m, int c0, int nn, const float* ia, int nga,
+                      const float* ib, int ngb, cudaStream_t s);
+}  // namespace ldist
+
 }  // namespace rg

@@ -66,6 +66,50 @@ def schedule(kernel, global_rows: int, cols: int, nranks: int, rank: int, iterat
     return out.asdict()
 
 
+def lud_layout(n: int, prow: int, pcol: int, rank: int):
+    """Host-only: (mloc, nloc), the local matrix shape of `rank` in rodinia_lud_dist's 2-D
+    block-cyclic layout (NB = 128 blocks, rank = pr * pcol + pc)."""
+    m, k = ctypes.c_int64(0), ctypes.c_int64(0)
+    check(lib.rodinia_lud_dist_layout(n, prow, pcol, rank, ctypes.byref(m), ctypes.byref(k)),
+          "rodinia_lud_dist_layout")
+    return m.value, k.value
+
+
+LUD_NB = 128
+
+
+def _bc_index(n: int, P: int, p: int):
+    """Global indices of the rows (or columns) of the blocks I = p (mod P), increasing I."""
+    import numpy as np
+    nb = (n + LUD_NB - 1) // LUD_NB
+    return np.concatenate([np.arange(I * LUD_NB, min(n, (I + 1) * LUD_NB)) for I in range(p, nb, P)] or
+                          [np.zeros(0, dtype=np.int64)])
+
+
+def block_cyclic_scatter(A, prow: int, pcol: int):
+    """Layout only: the prow*pcol local matrices of a global n x n tensor (rank order)."""
+    import torch
+    n = A.shape[0]
+    out = []
+    for r in range(prow * pcol):
+        ri = torch.as_tensor(_bc_index(n, prow, r // pcol), device=A.device)
+        ci = torch.as_tensor(_bc_index(n, pcol, r % pcol), device=A.device)
+        out.append(A[ri][:, ci].contiguous())
+    return out
+
+
+def block_cyclic_gather(parts, n: int, prow: int, pcol: int):
+    """Layout only: the global n x n tensor from the local matrices (rank order)."""
+    import torch
+    A = torch.empty((n, n), dtype=parts[0].dtype, device=parts[0].device)
+    for r, x in enumerate(parts):
+        ri = torch.as_tensor(_bc_index(n, prow, r // pcol), device=A.device)
+        ci = torch.as_tensor(_bc_index(n, pcol, r % pcol), device=A.device)
+        if len(ri) and len(ci):
+            A[ri[:, None], ci[None, :]] = x
+    return A
+
+
 class HaloComm:
     def __init__(self, handle, nranks: int, rank: int, local: bool):
         self.handle = handle
@@ -120,6 +164,15 @@ class HaloComm:
                                        None if coeffs is None else ctypes.byref(coeffs), _g(g),
                                        _stream(stream)), "rodinia_hotspot_dist")
         return out_local
+
+    def lud(self, a_local, n: int, prow: int, pcol: int, stream=None):
+        """2-D block-cyclic LU (rodinia_lud_dist): this rank's local matrix (LOCAL communicator:
+        the list of all ranks' local matrices), factored in place."""
+        import torch
+        a, keep = self._ptrs(a_local, torch.float32, "a")
+        check(lib.rodinia_lud_dist(self.handle, a, int(n), int(prow), int(pcol), _stream(stream)),
+              "rodinia_lud_dist")
+        return a_local
 
     def srad(self, J_local, global_rows: int, r1, r2, c1, c2, lam: float, niter: int, g=None,
              stream=None):

@@ -1,7 +1,8 @@
 """Multi-rank NCCL run of the row-slab layer: one process per visible GPU (P in {2, 4, 8} up
 to the device count), torch.distributed (NCCL) only for the bootstrap and the result gather,
 halos through the library's own ncclSend/ncclRecv (csrc/dist.cu).  Sharded == single-GPU bit
-for bit, with R not divisible by P.  Skipped with fewer than two GPUs
+for bit, with R not divisible by P; the 2-D block-cyclic LU
+(rodinia_lud_dist, §8(f) #3) on a prow x pcol grid equals the single-rank bits.  Skipped with fewer than two GPUs
 (the builder's boxes have one; the driver's 8-GPU tier runs it)."""
 import os
 import socket
@@ -56,6 +57,22 @@ def _worker(rank, ws, port, q):
                 ref = torch.from_numpy(J).cuda()
                 rg.rodinia_srad(ref, 400, 527, 3, 130, 0.5, 20, g=g[:4] + (1,) + g[5:])
                 ok = ok and bool(torch.equal(torch.cat(parts), ref))
+        # 2-D block-cyclic LU (rodinia_lud_dist): every grid gives the single-rank bits
+        nlu = 1100
+        prow = 1 if ws == 2 else 2
+        pcol = ws // prow
+        A = torch.from_numpy(synth.lud_rodinia_matrix(nlu)).cuda()
+        mine = rg.dist.block_cyclic_scatter(A, prow, pcol)[rank]
+        comm.lud(mine, nlu, prow, pcol)
+        gathered = [None] * ws
+        dist.all_gather_object(gathered, mine.cpu())
+        if rank == 0:
+            got = rg.dist.block_cyclic_gather([g.cuda() for g in gathered], nlu, prow, pcol)
+            one = rg.dist.HaloComm.local_slabs(1)
+            ref = A.clone()
+            one.lud([ref], nlu, 1, 1)
+            one.close()
+            ok = ok and bool(torch.equal(got, ref))
         torch.cuda.synchronize()
         comm.close()
         q.put((rank, "ok" if ok else "mismatch"))
