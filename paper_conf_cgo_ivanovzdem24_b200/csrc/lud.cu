@@ -834,7 +834,15 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
 // its k < j terms; products fused (FMA); quotients = IEEE quotients formed from the pivot's
 // correctly rounded reciprocal (div_rcp).
 constexpr int LD_NB = 128;
-constexpr int D128_LD = 132;                   // 16-byte aligned rows, conflict-free row reads
+constexpr int D128_LD = 140;                   // 16-byte rows; row-per-lane 128-bit reads conflict-free
+constexpr int D128_LT = 132;                   // transposed L sub-panel: LT[k][i]
+#ifdef RG_LUD_PROBE  // development timing probes (printf of clock64 phase stamps)
+#define LUD_PROBE(i) if (threadIdx.x == 0) pr[i] = clock64()
+#define LUD_PROBE_W(i) if (threadIdx.x == 32) pw[i] = clock64()
+#else
+#define LUD_PROBE(i)
+#define LUD_PROBE_W(i)
+#endif
 constexpr int D128_IMG = 128 * D128_LD;        // one 128 x 128 image padded to D128_LD
 constexpr size_t d128_mimg_floats() { return (size_t)2 * D128_IMG + 128; }
 
@@ -850,28 +858,18 @@ __device__ __forceinline__ float div_rcp(float a, float b, float rb) {
 }
 
 // Right-looking LU of the rs x rs leading part of a 32 x 32 block held one row per lane
-// (a[j] = element (lane, j)), one warp.  Step kk: lane kk publishes its final row through the
-// shared-memory buffer rowbuf (double-buffered, broadcast reads), lanes kk < i < rs form
-// l_ik = a_ik / u_kk and subtract l_ik u_kj for j > kk (others use l = 0: row unchanged).
+// (a[j] = element (lane, j)), one warp.  Step kk: row kk (final) is broadcast from lane kk
+// with warp shuffles, lanes kk < i < rs form l_ik = a_ik / u_kk and subtract l_ik u_kj for
+// j > kk (others use l = 0: row unchanged).
 // rinv[i] = RN(1/u_ii) for i < rs.
 __device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rowbuf, float* rinv) {
     float myrb = 0.f;
 #pragma unroll
     for (int kk = 0; kk < 32; ++kk) {
         if (kk >= rs) break;  // uniform
-        float* row = rowbuf + 32 * (kk & 1);
-        if (lane == kk) {
-#pragma unroll
-            for (int q = kk / 4; q < 8; ++q)
-                *reinterpret_cast<float4*>(row + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
-        }
-        __syncwarp();
         float u[32];
 #pragma unroll
-        for (int q = kk / 4; q < 8; ++q) {
-            const float4 t = *reinterpret_cast<const float4*>(row + 4 * q);
-            u[4 * q] = t.x; u[4 * q + 1] = t.y; u[4 * q + 2] = t.z; u[4 * q + 3] = t.w;
-        }
+        for (int j = kk; j < 32; ++j) u[j] = __shfl_sync(0xffffffffu, a[j], kk);  // row kk, broadcast
         const float rb = __frcp_rn(u[kk]);
         if (lane == kk) myrb = rb;
         const bool below = lane > kk && lane < rs;
@@ -881,6 +879,7 @@ __device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, 
         for (int j = kk + 1; j < 32; ++j) a[j] = __fmaf_rn(-l, u[j], a[j]);
     }
     if (lane < rs) rinv[lane] = myrb;
+    (void)rowbuf;
 }
 
 // One CTA of 256 threads factors the r x r block at A (r <= 128, row stride lda) in shared
@@ -892,12 +891,17 @@ __device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, 
 // L^T image | RN(1/u_jj)] (d128_mimg_floats), written with bulk copies.
 __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int lda, int r, float* __restrict__ mimg) {
     constexpr int LD = D128_LD;
-    extern __shared__ __align__(128) float S[];  // 132 x LD, then the transposed image 128 x LD
+    extern __shared__ __align__(128) float S[];  // 132 x LD, the transposed image 128 x LD, LT 32 x D128_LT
     __shared__ __align__(16) float rowbuf[64];
     __shared__ __align__(16) float rinv[128];
     __shared__ __align__(8) uint64_t mbar;
     float* T = S + 132 * LD;
+    float* LT = T + 128 * LD;  // the current sub-panel's L columns, transposed (rows >= r stay 0)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+#ifdef RG_LUD_PROBE
+    long long pr[16] = {0}, pw[16] = {0};
+#endif
+    LUD_PROBE(0);
     const bool bulk = r == 128 && (lda & 3) == 0 && ((uintptr_t)A & 15) == 0;
     if (bulk) {  // 128 row copies of 512 B
         if (tid == 0) {
@@ -920,12 +924,15 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
             S[i * LD + j] = v[q];
         }
     }
-    for (int e = tid; e < 4 * LD + 128 * 4; e += 256) {  // zero padding: rows 128..131, cols 128..131
+    constexpr int PADC = LD - 128;
+    for (int e = tid; e < 4 * LD + 128 * PADC; e += 256) {  // zero padding: rows 128..131, cols 128..LD-1
         if (e < 4 * LD) S[128 * LD + e] = 0.f;
-        else S[((e - 4 * LD) >> 2) * LD + 128 + ((e - 4 * LD) & 3)] = 0.f;
+        else S[((e - 4 * LD) / PADC) * LD + 128 + ((e - 4 * LD) % PADC)] = 0.f;
     }
+    for (int e = tid; e < 32 * D128_LT; e += 256) LT[e] = 0.f;
     if (bulk) tc::mbar_wait(&mbar, 0);
     __syncthreads();
+    LUD_PROBE(1);
     if (warp == 0) {  // the first diagonal sub-block
         float a[32];
 #pragma unroll
@@ -939,6 +946,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
             *reinterpret_cast<float4*>(S + lane * LD + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
     }
     __syncthreads();
+    LUD_PROBE(2);
 #pragma unroll 1
     for (int p = 0; p + 32 < r; p += 32) {
         const int rest = r - p - 32;  // rows below / columns right of the factored sub-block
@@ -967,6 +975,8 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(xr + 4 * q) = make_float4(x[4 * q], x[4 * q + 1], x[4 * q + 2], x[4 * q + 3]);
+#pragma unroll
+            for (int k = 0; k < 32; ++k) LT[k * D128_LT + p + 32 + tid] = x[k];
         } else if (tid >= 128 && tid - 128 < rest) {
             // U column c: y_i = a_ic - sum_{k<i} l_ik y_k (unit-lower sub-block)
             const int c = p + 32 + (tid - 128);
@@ -981,80 +991,85 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
             for (int i = 0; i < 32; ++i) S[(p + i) * LD + c] = y[i];
         }
         __syncthreads();
+        LUD_PROBE(3 + 3 * (p / 32));
         const int nb = p + 32;
+        {
+            // the next diagonal sub-block's rank-32 update first, by all threads (4 elements each)
+            const int i = nb + (tid >> 3), j0 = nb + 4 * (tid & 7);
+            float4 c = *reinterpret_cast<const float4*>(S + i * LD + j0);
+#pragma unroll 8
+            for (int k = 0; k < 32; ++k) {
+                const float l = -LT[k * D128_LT + i];
+                const float4 u = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
+                c.x = __fmaf_rn(l, u.x, c.x);
+                c.y = __fmaf_rn(l, u.y, c.y);
+                c.z = __fmaf_rn(l, u.z, c.z);
+                c.w = __fmaf_rn(l, u.w, c.w);
+            }
+            *reinterpret_cast<float4*>(S + i * LD + j0) = c;
+        }
+        __syncthreads();
         if (warp == 0) {
-            // the next diagonal sub-block: its rank-32 update, then its factorisation
-            float lr[32], a[32];
+            // ... then its factorisation, while the other warps update the rest
+            float a[32];
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
-                const float4 t = *reinterpret_cast<const float4*>(S + (nb + lane) * LD + p + 4 * q);
-                lr[4 * q] = -t.x; lr[4 * q + 1] = -t.y; lr[4 * q + 2] = -t.z; lr[4 * q + 3] = -t.w;
                 const float4 c = *reinterpret_cast<const float4*>(S + (nb + lane) * LD + nb + 4 * q);
                 a[4 * q] = c.x; a[4 * q + 1] = c.y; a[4 * q + 2] = c.z; a[4 * q + 3] = c.w;
             }
-#pragma unroll
-            for (int k = 0; k < 32; ++k) {
-                const float4* ur = reinterpret_cast<const float4*>(S + (p + k) * LD + nb);
-#pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const float4 u = ur[q];
-                    a[4 * q] = __fmaf_rn(lr[k], u.x, a[4 * q]);
-                    a[4 * q + 1] = __fmaf_rn(lr[k], u.y, a[4 * q + 1]);
-                    a[4 * q + 2] = __fmaf_rn(lr[k], u.z, a[4 * q + 2]);
-                    a[4 * q + 3] = __fmaf_rn(lr[k], u.w, a[4 * q + 3]);
-                }
-            }
+            LUD_PROBE(4 + 3 * (p / 32));
             diag32_factor(a, min(32, rest), lane, rowbuf, rinv + nb);
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(S + (nb + lane) * LD + nb + 4 * q) =
                     make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
         } else {
-            // rank-32 update of the rest of [nb, r)^2 (tiles may reach into the zero padding)
-            const int nt = (rest + 3) / 4;
-            for (int t = tid - 32; t < nt * nt; t += 224) {
-                const int ti = t / nt, tj = t - (t / nt) * nt;
-                if (ti < 8 && tj < 8) continue;  // the next diagonal sub-block (warp 0)
-                const int i0 = nb + 4 * ti, j0 = nb + 4 * tj;
-                float acc[4][4];
+            // rank-32 update of the rest of [nb, r)^2: units of 4 rows x 8 columns, consecutive lanes
+            // on consecutive row groups of one column group (u rows broadcast, LT rows 128-bit);
+            // units may reach into the zero padding (rows < 132, columns < LD): 0 - 0 * u
+            const int nrg = (rest + 3) / 4, ncg = (rest + 7) / 8;
+            for (int t = tid - 32; t < nrg * ncg; t += 224) {
+                const int cg = t / nrg, rg = t - cg * nrg;
+                if (rg < 8 && cg < 4) continue;  // the next diagonal sub-block (warp 0)
+                const int i0 = nb + 4 * rg, j0 = nb + 8 * cg;
+                float acc[4][8];
 #pragma unroll
                 for (int a = 0; a < 4; ++a) {
-                    const float4 v = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0);
-                    acc[a][0] = v.x; acc[a][1] = v.y; acc[a][2] = v.z; acc[a][3] = v.w;
+                    const float4 v0 = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0);
+                    const float4 v1 = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0 + 4);
+                    acc[a][0] = v0.x; acc[a][1] = v0.y; acc[a][2] = v0.z; acc[a][3] = v0.w;
+                    acc[a][4] = v1.x; acc[a][5] = v1.y; acc[a][6] = v1.z; acc[a][7] = v1.w;
                 }
-#pragma unroll 8
+#pragma unroll 4
                 for (int k = 0; k < 32; ++k) {
-                    const float4 u = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
+                    const float4 u0 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
+                    const float4 u1 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0 + 4);
+                    const float4 l4 = *reinterpret_cast<const float4*>(LT + k * D128_LT + i0);
+                    const float u[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+                    const float l[4] = {-l4.x, -l4.y, -l4.z, -l4.w};
 #pragma unroll
-                    for (int a = 0; a < 4; ++a) {
-                        const float l = -S[(i0 + a) * LD + p + k];
-                        acc[a][0] = __fmaf_rn(l, u.x, acc[a][0]);
-                        acc[a][1] = __fmaf_rn(l, u.y, acc[a][1]);
-                        acc[a][2] = __fmaf_rn(l, u.z, acc[a][2]);
-                        acc[a][3] = __fmaf_rn(l, u.w, acc[a][3]);
-                    }
+                    for (int a = 0; a < 4; ++a)
+#pragma unroll
+                        for (int b = 0; b < 8; ++b) acc[a][b] = __fmaf_rn(l[a], u[b], acc[a][b]);
                 }
 #pragma unroll
-                for (int a = 0; a < 4; ++a)
-                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0) =
-                        make_float4(acc[a][0], acc[a][1], acc[a][2], acc[a][3]);
+                for (int a = 0; a < 4; ++a) {
+                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0) = make_float4(acc[a][0], acc[a][1], acc[a][2], acc[a][3]);
+                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0 + 4) = make_float4(acc[a][4], acc[a][5], acc[a][6], acc[a][7]);
+                }
             }
+            LUD_PROBE_W(p / 32);
         }
         __syncthreads();
+        LUD_PROBE(5 + 3 * (p / 32));
     }
-    // outputs: the transposed image in shared memory, then bulk stores (A rows, images, 1/u)
-    for (int e = tid; e < 128 * 128; e += 256) {
-        const int i = e >> 7, k = e & 127;
-        T[k * LD + i] = S[i * LD + k];
-    }
-    for (int e = tid; e < 128 * 4; e += 256) T[(e >> 2) * LD + 128 + (e & 3)] = 0.f;
+    // outputs: bulk stores of the row-major image, 1/u and the A rows first, then the transposed
+    // image built in shared memory meanwhile
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncthreads();
     if (tid == 0) {
         asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg),
                      "r"(tc::smem_u32(S)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
-        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + D128_IMG),
-                     "r"(tc::smem_u32(T)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
         asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + 2 * D128_IMG),
                      "r"(tc::smem_u32(rinv)), "r"(512u) : "memory");
     }
@@ -1069,9 +1084,31 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
         }
     }
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    for (int e = tid; e < 128 * 128; e += 256) {
+        const int i = e >> 7, k = e & 127;
+        T[k * LD + i] = S[i * LD + k];
+    }
+    for (int e = tid; e < 128 * PADC; e += 256) T[(e / PADC) * LD + 128 + (e % PADC)] = 0.f;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    if (tid == 0) {
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + D128_IMG),
+                     "r"(tc::smem_u32(T)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    }
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // shared memory read before exit
+#ifdef RG_LUD_PROBE
+    LUD_PROBE(14);
+    if (tid == 32) printf("diag128 rest-update end (warp 1): %lld %lld %lld\n", pw[0], pw[1], pw[2]);
+    __syncthreads();
+    if (tid == 0)
+        printf("diag128 r=%d load %lld diag0 %lld | p0 LU %lld dupd %lld factor+rest %lld | p1 %lld %lld %lld | p2 %lld %lld %lld | "
+               "out %lld  [p0 start %lld]\n", r, pr[1] - pr[0], pr[2] - pr[1], pr[3] - pr[2], pr[4] - pr[3], pr[5] - pr[4],
+               pr[6] - pr[5], pr[7] - pr[6], pr[8] - pr[7], pr[9] - pr[8], pr[10] - pr[9], pr[11] - pr[10],
+               pr[14] - pr[11], pr[3]);
+#endif
 }
-constexpr size_t d128_smem() { return (size_t)(132 + 128) * D128_LD * sizeof(float); }
+constexpr size_t d128_smem() { return ((size_t)(132 + 128) * D128_LD + 32 * D128_LT) * sizeof(float); }
 
 // Triangular solves against the factored 128 x 128 diagonal block (mimg from lud_diag128),
 // 64 threads per CTA, one thread per row (lower: L = A U^-1, row t at A + t*lda) or per
