@@ -729,7 +729,10 @@ extern "C" rodinia_status rodinia_srad_dist(rodinia_comm* c, void* J_local, int6
 //   2. process column qk solves its L_Ik, process row pk its U_kJ (ldist::trsm), each writing
 //      the hi/lo operand image of its panel;
 //   3. L images travel along process rows, U images along process columns (send/recv);
-//   4. every rank updates its trailing blocks (ldist::update, tensor cores).
+//   4. every rank updates its trailing blocks (ldist::update, tensor cores): first the blocks of
+//      block row / column k+1 (the next step's panel, on the main stream), then the rest on a
+//      low-priority side stream, which runs under the next step's 1.-3. (look-ahead; the images
+//      are double-buffered by step parity, and the next step's updates wait for the rest).
 namespace rg {
 static int64_t bc_extent(int64_t n, int P, int p) {  // rows of the global blocks I = p (mod P)
     const int64_t nb = (n + ldist::NB - 1) / ldist::NB;
@@ -746,8 +749,8 @@ struct LudRank {
     int64_t mloc, nloc;
     float** slot;
     float* mimg;
-    float* ia;
-    float* ib;
+    float* ia[2];
+    float* ib[2];
 };
 }  // namespace rg
 
@@ -768,7 +771,7 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
         return set_error(RODINIA_E_INVALID, "lud_dist: process grid %d x %d != %d ranks", prow, pcol, c->nranks);
     if (n > (int64_t)1 << 20) return set_error(RODINIA_E_INVALID, "lud_dist: n too large");
     std::lock_guard<std::mutex> lk(c->mu);
-    cudaStream_t s = (cudaStream_t)stream;
+    cudaStream_t us = (cudaStream_t)stream;
     const int P = c->nranks;
     std::vector<LudRank> rk;
     for (int r = 0; r < P; ++r) {
@@ -781,35 +784,66 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
         x.A = (float*)arg_ptr(c, a_local, rk.size());
         x.mloc = bc_extent(n, prow, x.pr);
         x.nloc = bc_extent(n, pcol, x.pc);
+        if (x.mloc > 0 && x.nloc > 0 && !x.A) return set_error(RODINIA_E_INVALID, "lud_dist: null local matrix");
         rk.push_back(x);
     }
+    // streams: the main chain on a high-priority stream, the remainder updates on a low-priority
+    // side stream; both are joined to the caller's stream at entry and exit
+    int prio_lo = 0, prio_hi = 0;
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    cudaStream_t s = nullptr, s2 = nullptr;
+    cudaEvent_t ev_in = nullptr, ev_img = nullptr, ev_rest = nullptr;
+    RG_CUDA(cudaStreamCreateWithPriority(&s, cudaStreamNonBlocking, prio_hi));
+    RG_CUDA(cudaStreamCreateWithPriority(&s2, cudaStreamNonBlocking, prio_lo));
+    RG_CUDA(cudaEventCreateWithFlags(&ev_in, cudaEventDisableTiming));
+    RG_CUDA(cudaEventCreateWithFlags(&ev_img, cudaEventDisableTiming));
+    RG_CUDA(cudaEventCreateWithFlags(&ev_rest, cudaEventDisableTiming));
+    RG_CUDA(cudaEventRecord(ev_in, us));
+    RG_CUDA(cudaStreamWaitEvent(s, ev_in, 0));
+    RG_CUDA(cudaStreamWaitEvent(s2, ev_in, 0));
     auto cleanup = [&]() {
+        cudaEventRecord(ev_rest, s2);  // join the side stream, release the scratch, join the caller
+        cudaStreamWaitEvent(s, ev_rest, 0);
         for (auto& x : rk)
-            for (void* p : {(void*)x.slot, (void*)x.mimg, (void*)x.ia, (void*)x.ib})
+            for (void* p : {(void*)x.slot, (void*)x.mimg, (void*)x.ia[0], (void*)x.ia[1], (void*)x.ib[0],
+                            (void*)x.ib[1]})
                 if (p) cudaFreeAsync(p, s);
+        cudaEventRecord(ev_in, s);
+        cudaStreamWaitEvent(us, ev_in, 0);
+        cudaStreamDestroy(s);
+        cudaStreamDestroy(s2);
+        cudaEventDestroy(ev_in);
+        cudaEventDestroy(ev_img);
+        cudaEventDestroy(ev_rest);
     };
+    bool alloc_ok = true;
     for (auto& x : rk) {
-        if ((x.mloc > 0 && x.nloc > 0 && !x.A) ||
-            cudaMallocAsync((void**)&x.slot, sizeof(float*), s) != cudaSuccess ||
-            cudaMallocAsync((void**)&x.mimg, ldist::mimg_floats() * sizeof(float), s) != cudaSuccess ||
-            cudaMallocAsync((void**)&x.ia, ldist::img_floats(std::max<int64_t>(x.mloc, 1)) * sizeof(float), s) !=
-                cudaSuccess ||
-            cudaMallocAsync((void**)&x.ib, ldist::img_floats(std::max<int64_t>(x.nloc, 1)) * sizeof(float), s) !=
-                cudaSuccess) {
-            cudaGetLastError();
-            cleanup();
-            return set_error(RODINIA_E_NOMEM, "lud_dist: scratch allocation failed");
-        }
-        rodinia_status st = ldist::set_slot(x.slot, x.A, s);
+        const size_t fa = ldist::img_floats(std::max<int64_t>(x.mloc, 1));
+        const size_t fb = ldist::img_floats(std::max<int64_t>(x.nloc, 1));
+        alloc_ok = alloc_ok && cudaMallocAsync((void**)&x.slot, sizeof(float*), s) == cudaSuccess &&
+                   cudaMallocAsync((void**)&x.mimg, ldist::mimg_floats() * sizeof(float), s) == cudaSuccess;
+        for (int b = 0; b < 2; ++b)
+            alloc_ok = alloc_ok && cudaMallocAsync((void**)&x.ia[b], fa * sizeof(float), s) == cudaSuccess &&
+                       cudaMallocAsync((void**)&x.ib[b], fb * sizeof(float), s) == cudaSuccess;
+        if (!alloc_ok) break;
+    }
+    if (!alloc_ok) {
+        cudaGetLastError();
+        cleanup();
+        return set_error(RODINIA_E_NOMEM, "lud_dist: scratch allocation failed");
+    }
+    rodinia_status st = RODINIA_OK;
+    for (auto& x : rk) {
+        st = ldist::set_slot(x.slot, x.A, s);
         if (st != RODINIA_OK) { cleanup(); return st; }
     }
     NcclApi* api = nullptr;
     if (c->kind != 1 && P > 1) {
-        rodinia_status st = nccl_api(&api);
+        st = nccl_api(&api);
         if (st != RODINIA_OK) { cleanup(); return st; }
     }
     const int64_t NB = ldist::NB, nb = (n + NB - 1) / NB;
-    rodinia_status st = RODINIA_OK;
+    bool rest_pending = false;
     auto find = [&](int r) -> LudRank* {
         for (auto& x : rk)
             if (x.r == r) return &x;
@@ -820,11 +854,17 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
         st = (x);                        \
         if (st != RODINIA_OK) goto done; \
     } while (0)
+#define LD_CUDA(x, what)                                                                     \
+    do {                                                                                     \
+        cudaError_t _e = (x);                                                                \
+        if (_e != cudaSuccess) { st = cuda_error(_e, what, __FILE__, __LINE__); goto done; } \
+    } while (0)
     for (int64_t k = 0; k < nb; ++k) {
         const int pk = (int)(k % prow), qk = (int)(k % pcol), root = pk * pcol + qk;
         const int bk = (int)std::min<int64_t>(NB, n - k * NB);
         const int64_t lrk = (k / prow) * NB, lck = (k / pcol) * NB;  // block (k, k) on its owner
-        if (LudRank* o = find(root)) LD_TRY(ldist::diag(o->A + lrk * o->nloc + lck, (int)o->nloc, bk, o->mimg, s));
+        const int par = (int)(k & 1);
+        if (LudRank* o = find(root)) LD_TRY(ldist::diag(o->slot, (size_t)(lrk * o->nloc + lck), (int)o->nloc, bk, o->mimg, s));
         if (k == nb - 1) break;
         // 1. the diagonal block's images to every rank
         if (P > 1) {
@@ -833,22 +873,26 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
                 LudRank* o = find(root);
                 for (auto& x : rk)
                     if (x.r != root)
-                        if (cudaMemcpyAsync(x.mimg, o->mimg, cnt * sizeof(float), cudaMemcpyDeviceToDevice, s) !=
-                            cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist bcast", __FILE__, __LINE__); goto done; }
+                        LD_CUDA(cudaMemcpyAsync(x.mimg, o->mimg, cnt * sizeof(float), cudaMemcpyDeviceToDevice, s),
+                                "lud_dist bcast");
             } else {
                 ncclResult_t e = api->Bcast(rk[0].mimg, rk[0].mimg, cnt, ncclFloat32, root, c->nccl, s);
                 if (e != ncclSuccess) { st = set_error(RODINIA_E_NCCL, "lud_dist bcast: %s", api->GetErrorString(e)); goto done; }
             }
         }
-        // 2. panel solves: L_Ik on process column qk, U_kJ on process row pk
+        // 2. panel solves into this step's images (the side stream's remainder update of step
+        //    k-2 read them; the main stream waited for it before step k-1's updates)
         for (auto& x : rk) {
             const int64_t lr0 = bc_blocks_le(k, prow, x.pr) * NB, lc0 = bc_blocks_le(k, pcol, x.pc) * NB;
+            ldist::TrsmJob jobs[2];
+            int nj = 0;
             if (x.pc == qk && x.mloc > lr0)
-                LD_TRY(ldist::trsm(x.A + lr0 * x.nloc + lck, (int)x.nloc, true, (int)(x.mloc - lr0), x.ia,
-                                   ldist::img_groups(x.mloc - lr0), x.mimg, s));
+                jobs[nj++] = ldist::TrsmJob{x.slot, (size_t)(lr0 * x.nloc + lck), (int)x.nloc, 1, (int)(x.mloc - lr0), x.ia[par],
+                                            ldist::img_groups(x.mloc - lr0)};
             if (x.pr == pk && x.nloc > lc0)
-                LD_TRY(ldist::trsm(x.A + lrk * x.nloc + lc0, (int)x.nloc, false, (int)(x.nloc - lc0), x.ib,
-                                   ldist::img_groups(x.nloc - lc0), x.mimg, s));
+                jobs[nj++] = ldist::TrsmJob{x.slot, (size_t)(lrk * x.nloc + lc0), (int)x.nloc, 0, (int)(x.nloc - lc0), x.ib[par],
+                                            ldist::img_groups(x.nloc - lc0)};
+            LD_TRY(ldist::trsm(jobs, nj, x.mimg, s));
         }
         // 3. L images along process rows (from (pr, qk)), U images along process columns (from (pk, pc))
         if (P > 1) {
@@ -856,16 +900,14 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
                 for (auto& x : rk) {
                     const int64_t rows = x.mloc - bc_blocks_le(k, prow, x.pr) * NB;
                     const int64_t cols = x.nloc - bc_blocks_le(k, pcol, x.pc) * NB;
-                    if (x.pc != qk && rows > 0) {
-                        LudRank* src = find(x.pr * pcol + qk);
-                        if (cudaMemcpyAsync(x.ia, src->ia, ldist::img_floats(rows) * sizeof(float),
-                                            cudaMemcpyDeviceToDevice, s) != cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist L image", __FILE__, __LINE__); goto done; }
-                    }
-                    if (x.pr != pk && cols > 0) {
-                        LudRank* src = find(pk * pcol + x.pc);
-                        if (cudaMemcpyAsync(x.ib, src->ib, ldist::img_floats(cols) * sizeof(float),
-                                            cudaMemcpyDeviceToDevice, s) != cudaSuccess) { st = cuda_error(cudaGetLastError(), "lud_dist U image", __FILE__, __LINE__); goto done; }
-                    }
+                    if (x.pc != qk && rows > 0)
+                        LD_CUDA(cudaMemcpyAsync(x.ia[par], find(x.pr * pcol + qk)->ia[par],
+                                                ldist::img_floats(rows) * sizeof(float), cudaMemcpyDeviceToDevice, s),
+                                "lud_dist L image");
+                    if (x.pr != pk && cols > 0)
+                        LD_CUDA(cudaMemcpyAsync(x.ib[par], find(pk * pcol + x.pc)->ib[par],
+                                                ldist::img_floats(cols) * sizeof(float), cudaMemcpyDeviceToDevice, s),
+                                "lud_dist U image");
                 }
             } else {
                 LudRank& x = rk[0];
@@ -876,18 +918,18 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
                     const size_t cnt = ldist::img_floats(rows);
                     if (x.pc == qk) {
                         for (int q = 0; q < pcol && e == ncclSuccess; ++q)
-                            if (q != qk) e = api->Send(x.ia, cnt, ncclFloat32, x.pr * pcol + q, c->nccl, s);
+                            if (q != qk) e = api->Send(x.ia[par], cnt, ncclFloat32, x.pr * pcol + q, c->nccl, s);
                     } else if (e == ncclSuccess) {
-                        e = api->Recv(x.ia, cnt, ncclFloat32, x.pr * pcol + qk, c->nccl, s);
+                        e = api->Recv(x.ia[par], cnt, ncclFloat32, x.pr * pcol + qk, c->nccl, s);
                     }
                 }
                 if (cols > 0 && prow > 1 && e == ncclSuccess) {
                     const size_t cnt = ldist::img_floats(cols);
                     if (x.pr == pk) {
                         for (int p = 0; p < prow && e == ncclSuccess; ++p)
-                            if (p != pk) e = api->Send(x.ib, cnt, ncclFloat32, p * pcol + x.pc, c->nccl, s);
+                            if (p != pk) e = api->Send(x.ib[par], cnt, ncclFloat32, p * pcol + x.pc, c->nccl, s);
                     } else {
-                        e = api->Recv(x.ib, cnt, ncclFloat32, pk * pcol + x.pc, c->nccl, s);
+                        e = api->Recv(x.ib[par], cnt, ncclFloat32, pk * pcol + x.pc, c->nccl, s);
                     }
                 }
                 ncclResult_t e2 = api->GroupEnd();
@@ -895,17 +937,33 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
                 if (e != ncclSuccess) { st = set_error(RODINIA_E_NCCL, "lud_dist panels: %s", api->GetErrorString(e)); goto done; }
             }
         }
-        // 4. local trailing updates
-        for (auto& x : rk) {
-            const int64_t lr0 = bc_blocks_le(k, prow, x.pr) * NB, lc0 = bc_blocks_le(k, pcol, x.pc) * NB;
-            const int64_t rows = x.mloc - lr0, cols = x.nloc - lc0;
-            if (rows > 0 && cols > 0)
-                LD_TRY(ldist::update(x.slot, (int)x.nloc, (int)lr0, (int)rows, (int)lc0, (int)cols, x.ia,
-                                     ldist::img_groups(rows), x.ib, ldist::img_groups(cols), s));
+        // 4. trailing updates: block row / column k+1 now (main), the rest on the side stream
+        LD_CUDA(cudaEventRecord(ev_img, s), "lud_dist event");
+        if (rest_pending) LD_CUDA(cudaStreamWaitEvent(s, ev_rest, 0), "lud_dist event");
+        LD_CUDA(cudaStreamWaitEvent(s2, ev_img, 0), "lud_dist event");
+        {
+            const int pn = (int)((k + 1) % prow), qn = (int)((k + 1) % pcol);
+            for (auto& x : rk) {
+                const int64_t lr0 = bc_blocks_le(k, prow, x.pr) * NB, lc0 = bc_blocks_le(k, pcol, x.pc) * NB;
+                const int64_t rows = x.mloc - lr0, cols = x.nloc - lc0;
+                if (rows <= 0 || cols <= 0) continue;
+                // block row / column k+1 are this rank's first trailing local block row / column
+                const int64_t mb = x.pr == pn ? std::min<int64_t>(NB, rows) : 0;
+                const int64_t nbk = x.pc == qn ? std::min<int64_t>(NB, cols) : 0;
+                const int ga = ldist::img_groups(rows), gb = ldist::img_groups(cols);
+                const int next[2][4] = {{(int)lr0, (int)rows, (int)lc0, (int)nbk},                 // column k+1
+                                        {(int)lr0, (int)mb, (int)(lc0 + nbk), (int)(cols - nbk)}};  // row k+1
+                LD_TRY(ldist::update(x.slot, (int)x.nloc, next, 2, (int)lr0, x.ia[par], ga, (int)lc0, x.ib[par], gb, s));
+                const int rest[1][4] = {{(int)(lr0 + mb), (int)(rows - mb), (int)(lc0 + nbk), (int)(cols - nbk)}};
+                LD_TRY(ldist::update(x.slot, (int)x.nloc, rest, 1, (int)lr0, x.ia[par], ga, (int)lc0, x.ib[par], gb, s2));
+            }
         }
+        LD_CUDA(cudaEventRecord(ev_rest, s2), "lud_dist event");
+        rest_pending = true;
     }
 done:
 #undef LD_TRY
+#undef LD_CUDA
     cleanup();
     return st;
 }

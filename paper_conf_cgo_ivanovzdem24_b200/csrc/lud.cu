@@ -20,6 +20,7 @@
 // the call sets first, so one graph serves every matrix of that size.
 #include <cuda_runtime.h>
 #include <string.h>
+#include <cstdlib>
 
 #include <algorithm>
 #include <map>
@@ -57,23 +58,14 @@ __global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, 
 // each own one column of U12 = L11^-1 A12 (forward substitution, unit-lower L11), lanes
 // P..2P-1 each own one row of L21 = A21 U11^-1.  Tiles are staged through shared memory with
 // coalesced loads, the substitutions run in registers with L11/U11 read by broadcast.
-// Panel-128 path (IMG): the kernel also writes its U12 columns / L21 rows, as the hi/lo TF32
-// parts of the tensor-core operand images, into the outer block's images (rows / columns from
-// `base`, k index kap0 + i): the images tc_split would build from the same final values.
-struct PerimImg {
-    float* a;   // A image (L21 rows)
-    float* b;   // B image (U12 columns, K-major)
-    int base, kap0, ng;
-};
-
 // Threads [0, P) own the U12 columns (unit-lower solve with L11 = dia's strict lower part),
 // threads [P, 2P) the L21 rows (solve with U11, then divide by the pivot).  Both are the same
 // loop over a row-major matrix M (L11 itself, or U11 transposed) whose rows are read four at a
 // time with 128-bit shared loads; per element the subtractions run in ascending j exactly as in
 // the two separate loops this replaces (same bits), with half the code (the fully unrolled pair
 // of solves overflowed the instruction cache: "no instruction" was the top stall, ncu r02f).
-template <int P, bool IMG>
-__device__ __forceinline__ void lud_perim_body(float* A, int n, int k, const PerimImg& im) {
+template <int P>
+__device__ __forceinline__ void lud_perim_body(float* A, int n, int k) {
     constexpr int LD = P + 4;  // 16-byte aligned rows
     __shared__ __align__(16) float msm[2][P][LD];  // [0]: L11 = dia (row-major), [1]: U11^T
     __shared__ float tile[2][P][P + 1];            // [0]: row tile A12, [1]: column tile A21
@@ -118,25 +110,14 @@ __device__ __forceinline__ void lud_perim_body(float* A, int n, int k, const Per
 #pragma unroll
             for (int i = 0; i < P; ++i) A[(size_t)(tb + lane) * n + o + i] = v[i];
         }
-        if constexpr (IMG) {
-            float* img = half == 0 ? im.b : im.a;
-#pragma unroll
-            for (int q = 0; q < P / 4; ++q) {
-                const float f[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
-                tc::img_store4(img, im.ng, tb + lane - im.base, im.kap0 + 4 * q, f);
-            }
-        }
     }
 }
 
 template <int P>
 __global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
-    lud_perim_body<P, false>(*slot, n, k, PerimImg{});
+    lud_perim_body<P>(*slot, n, k);
 }
 
-__global__ void __launch_bounds__(64) lud_perim_img(float* const* __restrict__ slot, int n, int k, PerimImg im) {
-    lud_perim_body<32, true>(*slot, n, k, im);
-}
 
 // ------------------------------------------------------------------ trailing update
 // The CTA stages by L21 tiles and bx U12 tiles in shared memory and walks its bx*by trailing
@@ -385,9 +366,10 @@ __global__ void __launch_bounds__(256)
 }
 
 namespace tc {
-// Launch helpers for the captured panel-128 factorisation: every kernel of the latency chain
-// (diagonal, panel, restricted updates) carries the highest launch priority, so that in the
-// graph it is scheduled ahead of the concurrently running trailing GEMM's CTAs.
+// Launch helper for the captured panel-128 factorisation: every kernel of the latency chain
+// (diagonal block, panel solves, next block's update) carries the highest launch priority, so
+// that in the graph (instantiated with cudaGraphInstantiateFlagUseNodePriority) it is scheduled
+// ahead of the concurrently running remainder update's CTAs.
 struct Lnch {
     cudaStream_t s;
     int prio;   // cudaLaunchAttributePriority value (0 = default)
@@ -407,79 +389,47 @@ inline void launch_p(const Lnch& L, void (*fn)(KArgs...), dim3 grid, dim3 block,
     cudaLaunchKernelEx(&cfg, fn, (KArgs)args...);
 }
 
-inline int update_img(const Lnch& L, float* const* slot, int n, const Rect* rs, int nr, const Img& im, int diag0) {
-    Args a;
-    a.nrect = 0;
-    for (int i = 0; i < nr; ++i)
-        if (rs[i].m > 0 && rs[i].nn > 0 && rs[i].kk > 0) a.rect[a.nrect++] = rs[i];
-    if (a.nrect == 0) return 0;
-    if (a.nrect == 1) a.rect[1] = a.rect[0];
-    const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
-    launch_p(L, lud_tc_update2, dim3(grid), dim3(128), smem_bytes2(), slot, n, a, im, diag0);
-    return 1;
-}
-
-// Whole factorisation, 128-wide outer blocks (inner panel 32), with look-ahead.  Returns the
-// launch count.  imgs: 4 images of img_floats(n) floats (A and B for two outer blocks).
-//  main branch (cs, high priority), per outer block [o, e):
-//    for each inner panel p0 = o + 32j: lud_diag<32>; lud_perim_img (U12/L21 + their hi/lo
-//    operand images, K chunks 2j, 2j+1 of the block's image); the rank-32 update of the block's
-//    L-shaped panel region from those chunks;
-//    then the part of the rank-128 trailing update that the NEXT block's panel needs (rows
-//    [e, e2) x cols [e, n) and rows [e2, n) x cols [e, e2), e2 = e + 128), after the previous
-//    block's remainder update (same region of C);
-//  side branch (cs2): the remainder of the rank-128 update, rows/cols [e2, n), which runs
-//    concurrently with the next block's panel chain (disjoint parts of C; the images are
-//    double-buffered by block parity).
-inline int launch_all(float* const* slot, int n, float* const imgs[4], cudaStream_t cs, cudaStream_t cs2,
-                      cudaEvent_t ev_fork, cudaEvent_t ev_img, cudaEvent_t ev_rest, int prio_hi) {
-    constexpr int NB = 128, P = 32;
-    const int m32 = (n + P - 1) / P;
+// v3 (round 2): the 1 x 1 case of the 2-D block-cyclic algorithm (ldist, DESIGN.md §5/§6) with
+// look-ahead.  Per 128-wide block column k, main branch (high priority): lud_diag128 factors
+// A_kk -> lud_trsm128 solves L21 and U12 in one launch, writing the operand images (double-
+// buffered by k's parity) -> the rank-128 update of block row / column k+1 (after the previous
+// remainder); side branch: the remainder update [e2, n)^2, concurrent with the next block's
+// diag/trsm.  Returns the launch count.
+inline int launch_all3(float* const* slot, int n, float* const imgs[4], float* mimg, cudaStream_t cs, cudaStream_t cs2,
+                       cudaEvent_t ev_fork, cudaEvent_t ev_img, cudaEvent_t ev_rest, int prio_hi) {
+    constexpr int NB = ldist::NB;
     int launches = 0;
-    const Lnch H{cs, prio_hi}, S{cs2, 0};
     cudaEventRecord(ev_fork, cs);
-    cudaStreamWaitEvent(cs2, ev_fork, 0);  // fork the side branch into the capture
+    cudaStreamWaitEvent(cs2, ev_fork, 0);
+    const int nb = (n + NB - 1) / NB;
     bool rest_pending = false;
-    for (int o = 0, blk = 0; o < n; o += NB, ++blk) {
-        const int e = std::min(n, o + NB);
-        const int base = std::min(o + P, n);
-        const int ng = ((n - base + 127) / 128 + 1) * 16;
-        float* ia = imgs[2 * (blk & 1)];
-        float* ib = imgs[2 * (blk & 1) + 1];
-        const Img im{ia, ib, base, base, ng, ng, 0};
-        for (int k = o / P; k * P < e; ++k) {
-            if (k == 0) {  // every later diagonal tile is factored by the update that precedes it
-                launch_p(H, lud_diag<P>, dim3(1), dim3(32), 0, slot, n, k);
-                ++launches;
-            }
-            if (k == m32 - 1) break;
-            const int j = k - o / P;
-            launch_p(H, lud_perim_img, dim3(m32 - k - 1), dim3(2 * P), 0, slot, n, k, PerimImg{ia, ib, base, P * j, ng});
+    for (int k = 0; k < nb; ++k) {
+        const int o = k * NB, bk = std::min(NB, n - o);
+        ldist::diag(slot, (size_t)o * n + o, n, bk, mimg, cs, prio_hi);
+        ++launches;
+        if (k == nb - 1) break;
+        const int e = o + NB, rows = n - e, ng = ldist::img_groups(rows);
+        float* ia = imgs[2 * (k & 1)];
+        float* ib = imgs[2 * (k & 1) + 1];
+        const ldist::TrsmJob jobs[2] = {{slot, (size_t)e * n + o, n, 1, rows, ia, ng},
+                                        {slot, (size_t)o * n + e, n, 0, rows, ib, ng}};
+        ldist::trsm(jobs, 2, mimg, cs, prio_hi);
+        ++launches;
+        cudaEventRecord(ev_img, cs);
+        if (rest_pending) cudaStreamWaitEvent(cs, ev_rest, 0);
+        cudaStreamWaitEvent(cs2, ev_img, 0);
+        const int e2 = std::min(n, e + NB), mb = e2 - e;
+        const int next[2][4] = {{e, rows, e, mb}, {e, mb, e2, n - e2}};  // block column / row k+1
+        ldist::update(slot, n, next, 2, e, ia, ng, e, ib, ng, cs, prio_hi);
+        ++launches;
+        if (e2 < n) {
+            const int rest[1][4] = {{e2, n - e2, e2, n - e2}};
+            ldist::update(slot, n, rest, 1, e, ia, ng, e, ib, ng, cs2, 0);
             ++launches;
-            const int p0 = k * P, a = p0 + P;  // inner panel columns [p0, a)
-            if (a < e) {
-                // rank-32 update restricted to the outer block's L-shaped panel region
-                const Rect rs[2] = {make_rect(a, a, n - a, e - a, p0, P), make_rect(a, e, e - a, n - e, p0, P)};
-                Img ij = im;
-                ij.c0 = 2 * j;
-                launches += update_img(H, slot, n, rs, 2, ij, a);  // + diagonal tile of step k+1
-            }
-        }
-        if (e < n) {  // rank-128 trailing update on the tensor cores, split for look-ahead
-            const int e2 = std::min(n, e + NB);
-            cudaEventRecord(ev_img, cs);  // this block's images are complete
-            if (rest_pending) cudaStreamWaitEvent(cs, ev_rest, 0);
-            const Rect rs[2] = {make_rect(e, e, e2 - e, n - e, o, e - o), make_rect(e2, e, n - e2, e2 - e, o, e - o)};
-            launches += update_img(H, slot, n, rs, 2, im, e);  // + diagonal tile of the next block
-            if (e2 < n) {
-                cudaStreamWaitEvent(cs2, ev_img, 0);
-                const Rect rr = make_rect(e2, e2, n - e2, n - e2, o, e - o);
-                launches += update_img(S, slot, n, &rr, 1, im, -1);
-                cudaEventRecord(ev_rest, cs2);
-                rest_pending = true;
-            } else {
-                rest_pending = false;
-            }
+            cudaEventRecord(ev_rest, cs2);
+            rest_pending = true;
+        } else {
+            rest_pending = false;
         }
     }
     cudaEventRecord(ev_rest, cs2);
@@ -633,24 +583,28 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         if (!ge.slot) RG_CUDA(cudaMalloc(&ge.slot, sizeof(float*)));
         const void* ifn = pl.tc ? (const void*)tc::lud_tc_update2
                                 : pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
-        if (pl.tc && !ge.img) RG_CUDA(cudaMalloc(&ge.img, 4 * tc::img_floats(n) * sizeof(float)));
+        const size_t fimg = std::max(tc::img_floats(n), ldist::img_floats(n));
+        if (pl.tc && !ge.img)  // 4 operand images + the diagonal-block payload (v3)
+            RG_CUDA(cudaMalloc(&ge.img, (4 * fimg + ldist::mimg_floats()) * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
         cudaStream_t cs, cs2;
         cudaEvent_t ev[3];
-        RG_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
-        RG_CUDA(cudaStreamCreateWithFlags(&cs2, cudaStreamNonBlocking));
-        for (auto& x : ev) RG_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+        // the capture stream carries the high priority (the panel-128 chain's kernel nodes inherit
+        // it); the side branch the low one
+        RG_CUDA(cudaStreamCreateWithPriority(&cs, cudaStreamNonBlocking, pl.tc ? prio_hi : prio_lo));
+        RG_CUDA(cudaStreamCreateWithPriority(&cs2, cudaStreamNonBlocking, prio_lo));
+        for (auto& x : ev) RG_CUDA(cudaEventCreateWithFlags(&x, cudaEventDisableTiming));
         cudaGraph_t graph;
         RG_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
         lud_set_slot<<<1, 1, 0, cs>>>(ge.slot, a);  // root node; argument replaced per launch
         int nl = 3 * m - 2;
         if (pl.tc) {
-            const size_t f = tc::img_floats(n);
+            const size_t f = fimg;
             float* const imgs[4] = {ge.img, ge.img + f, ge.img + 2 * f, ge.img + 3 * f};
-            nl = tc::launch_all(ge.slot, n, imgs, cs, cs2, ev[0], ev[1], ev[2], prio_hi);
+            nl = tc::launch_all3(ge.slot, n, imgs, ge.img + 4 * f, cs, cs2, ev[0], ev[1], ev[2], prio_hi);
         } else {
             launch_all(pl, ge.slot, n, cs);
         }
@@ -664,7 +618,8 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         e = cudaGraphGetRootNodes(graph, &root, &nroot);
         if (e == cudaSuccess && nroot == 1) e = cudaGraphKernelNodeGetParams(root, &ge.rootp);
         else if (e == cudaSuccess) e = cudaErrorInvalidValue;
-        if (e == cudaSuccess) e = cudaGraphInstantiate(&ge.exec, graph, 0);
+        // per-node launch priorities (the panel-128 chain) only take effect with this flag
+        if (e == cudaSuccess) e = cudaGraphInstantiateWithFlags(&ge.exec, graph, cudaGraphInstantiateFlagUseNodePriority);
         if (e != cudaSuccess) {
             ge.exec = nullptr;
             cudaGraphDestroy(graph);
@@ -862,7 +817,7 @@ __device__ __forceinline__ float div_rcp(float a, float b, float rb) {
 // with warp shuffles, lanes kk < i < rs form l_ik = a_ik / u_kk and subtract l_ik u_kj for
 // j > kk (others use l = 0: row unchanged).
 // rinv[i] = RN(1/u_ii) for i < rs.
-__device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rowbuf, float* rinv) {
+__device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rinv) {
     float myrb = 0.f;
 #pragma unroll
     for (int kk = 0; kk < 32; ++kk) {
@@ -879,7 +834,6 @@ __device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, 
         for (int j = kk + 1; j < 32; ++j) a[j] = __fmaf_rn(-l, u[j], a[j]);
     }
     if (lane < rs) rinv[lane] = myrb;
-    (void)rowbuf;
 }
 
 // One CTA of 256 threads factors the r x r block at A (r <= 128, row stride lda) in shared
@@ -889,10 +843,11 @@ __device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, 
 // diagonal sub-block and factors it (diag32_factor) while warps 1..7 update the rest of the
 // trailing block (4 x 4 register tiles).  Outputs: the block in A, and mimg = [U image |
 // L^T image | RN(1/u_jj)] (d128_mimg_floats), written with bulk copies.
-__global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int lda, int r, float* __restrict__ mimg) {
+__global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__ slot, size_t off, int lda, int r,
+                                                      float* __restrict__ mimg) {
+    float* A = *slot + off;  // the matrix pointer comes from a device slot (graph reuse, lud::run)
     constexpr int LD = D128_LD;
     extern __shared__ __align__(128) float S[];  // 132 x LD, the transposed image 128 x LD, LT 32 x D128_LT
-    __shared__ __align__(16) float rowbuf[64];
     __shared__ __align__(16) float rinv[128];
     __shared__ __align__(8) uint64_t mbar;
     float* T = S + 132 * LD;
@@ -940,7 +895,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
             const float4 t = *reinterpret_cast<const float4*>(S + lane * LD + 4 * q);
             a[4 * q] = t.x; a[4 * q + 1] = t.y; a[4 * q + 2] = t.z; a[4 * q + 3] = t.w;
         }
-        diag32_factor(a, min(32, r), lane, rowbuf, rinv);
+        diag32_factor(a, min(32, r), lane, rinv);
 #pragma unroll
         for (int q = 0; q < 8; ++q)
             *reinterpret_cast<float4*>(S + lane * LD + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
@@ -1018,7 +973,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* __restrict__ A, int
                 a[4 * q] = c.x; a[4 * q + 1] = c.y; a[4 * q + 2] = c.z; a[4 * q + 3] = c.w;
             }
             LUD_PROBE(4 + 3 * (p / 32));
-            diag32_factor(a, min(32, rest), lane, rowbuf, rinv + nb);
+            diag32_factor(a, min(32, rest), lane, rinv + nb);
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(S + (nb + lane) * LD + nb + 4 * q) =
@@ -1146,15 +1101,24 @@ __device__ __forceinline__ void trsm_load(const float* A, int lda, bool lower, b
     }
 }
 
-__global__ void __launch_bounds__(TR_T) lud_trsm128(float* __restrict__ A, int lda, int lower_, int count,
-                                                   float* __restrict__ img, int ng, const float* __restrict__ mimg) {
+// blockIdx.y selects one of (up to) two jobs of one launch (the owner of A_kk solves both its L
+// rows and its U columns at once); CTAs past a job's count exit.
+struct TrsmJobs {
+    ldist::TrsmJob j[2];
+};
+__global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* __restrict__ mimg) {
     constexpr int LD = D128_LD;
     extern __shared__ __align__(128) float sm[];
     __shared__ __align__(8) uint64_t mbar;
+    const ldist::TrsmJob& jb = jobs.j[blockIdx.y];
+    if ((int)blockIdx.x * TR_T >= jb.count) return;
+    float* __restrict__ A = *jb.slot + jb.off;
+    const int lda = jb.lda, count = jb.count, ng = jb.ng;
+    float* __restrict__ img = jb.img;
     float* M = sm;
     float* rinv = sm + D128_IMG;
     float* R = rinv + 128;
-    const bool lower = lower_ != 0;
+    const bool lower = jb.lower != 0;
     const int tid = threadIdx.x, idx = blockIdx.x * TR_T + tid;
     const bool own = idx < count;
     const bool vec = (lda & 3) == 0 && ((uintptr_t)A & 15) == 0;
@@ -1232,28 +1196,36 @@ size_t mimg_floats() { return d128_mimg_floats(); }
 int img_groups(int64_t rows) { return (int)(((rows + 127) / 128 + 1) * 16); }
 size_t img_floats(int64_t rows) { return (size_t)16 * img_groups(rows) * tc::KC2 * 8; }
 
-rodinia_status diag(float* A, int lda, int r, float* mimg, cudaStream_t s) {
+rodinia_status diag(float* const* slot, size_t off, int lda, int r, float* mimg, cudaStream_t s, int prio) {
     static bool attr = false;
     if (!attr) {
         RG_CUDA(cudaFuncSetAttribute((const void*)lud_diag128, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)d128_smem()));
         attr = true;
     }
-    lud_diag128<<<1, 256, d128_smem(), s>>>(A, lda, r, mimg);
+    tc::launch_p(tc::Lnch{s, prio}, lud_diag128, dim3(1), dim3(256), d128_smem(), slot, off, lda, r, mimg);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;
 }
 
-rodinia_status trsm(float* A, int lda, bool lower, int count, float* img, int ng, const float* mimg, cudaStream_t s) {
+rodinia_status trsm(const TrsmJob* job, int njobs, const float* mimg, cudaStream_t s, int prio) {
     static bool attr = false;
     if (!attr) {
         RG_CUDA(cudaFuncSetAttribute((const void*)lud_trsm128, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)trsm_smem()));
         attr = true;
     }
-    if (count <= 0) return RODINIA_OK;
-    lud_trsm128<<<(count + TR_T - 1) / TR_T, TR_T, trsm_smem(), s>>>(A, lda, lower ? 1 : 0, count, img, ng, mimg);
+    TrsmJobs js;
+    memset(&js, 0, sizeof js);
+    int nj = 0, cmax = 0;
+    for (int i = 0; i < njobs && i < 2; ++i)
+        if (job[i].count > 0) {
+            js.j[nj++] = job[i];
+            cmax = std::max(cmax, job[i].count);
+        }
+    if (nj == 0) return RODINIA_OK;
+    tc::launch_p(tc::Lnch{s, prio}, lud_trsm128, dim3((cmax + TR_T - 1) / TR_T, nj), dim3(TR_T), trsm_smem(), js, mimg);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;
@@ -1265,21 +1237,24 @@ rodinia_status set_slot(float** slot, float* a, cudaStream_t s) {
     return RODINIA_OK;
 }
 
-rodinia_status update(float* const* slot, int lda, int r0, int m, int c0, int nn, const float* ia, int nga,
-                      const float* ib, int ngb, cudaStream_t s) {
+rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr, int a_base, const float* ia,
+                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio) {
     static bool attr = false;
     if (!attr) {
         RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update2, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)tc::smem_bytes2()));
         attr = true;
     }
-    if (m <= 0 || nn <= 0) return RODINIA_OK;
     tc::Args a;
-    a.nrect = 1;
-    a.rect[0] = tc::make_rect(r0, c0, m, nn, 0, LD_NB);
-    a.rect[1] = a.rect[0];
-    const tc::Img im{ia, ib, r0, c0, nga, ngb, 0};
-    tc::lud_tc_update2<<<a.rect[0].tiles, 128, tc::smem_bytes2(), s>>>(slot, lda, a, im, -1);
+    a.nrect = 0;
+    for (int i = 0; i < nr && i < 2; ++i)  // rect[i] = {r0, m, c0, nn}
+        if (rect[i][1] > 0 && rect[i][3] > 0)
+            a.rect[a.nrect++] = tc::make_rect(rect[i][0], rect[i][2], rect[i][1], rect[i][3], 0, LD_NB);
+    if (a.nrect == 0) return RODINIA_OK;
+    if (a.nrect == 1) a.rect[1] = a.rect[0];
+    const tc::Img im{ia, ib, a_base, b_base, nga, ngb, 0};
+    const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
+    tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update2, dim3(grid), dim3(128), tc::smem_bytes2(), slot, lda, a, im);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;

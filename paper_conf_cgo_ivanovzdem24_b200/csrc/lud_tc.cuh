@@ -8,15 +8,13 @@
 
 namespace rg {
 // ------------------------------------------------------------------ tensor-core trailing update
-// Panel width 128 (DESIGN.md §5 "lud on tensor cores").  Two-level blocking:
-// every 128-wide outer block runs the panel-32 steps (lud_diag<32>, lud_perim<32>) with their
-// rank-32 updates restricted to the outer block's L-shaped panel region, then ONE rank-128
-// update of the trailing matrix A22 -= L21 * U12 on the 5th-generation tensor cores
-// (tcgen05.mma kind::tf32, accumulator in TMEM).  fp32 accuracy comes from the 3xTF32 split:
-// x = hi + lo with hi = x with its 13 low mantissa bits cleared (exactly a TF32 value) and
-// lo = x - hi (exact in fp32); A*B ~ hi*hi + hi*lo + lo*hi, dropping lo*lo (relative 2^-22)
-// and the TF32 truncation of lo (relative 2^-21).  The inner rank-32 updates use the same
-// kernel with K = 32.
+// Panel width 128 (DESIGN.md §5 "lud on tensor cores"): per 128-wide block
+// column, the diagonal block and the L21 / U12 panels are factored / solved by lud_diag128 and
+// lud_trsm128 (lud.cu), then ONE rank-128 update of the trailing matrix A22 -= L21 * U12 runs
+// on the 5th-generation tensor cores (tcgen05.mma kind::tf32, accumulator in TMEM).  fp32
+// accuracy comes from the 3xTF32 split: x = hi + lo with hi = x with its 13 low mantissa bits
+// cleared (exactly a TF32 value) and lo = x - hi (exact in fp32); A*B ~ hi*hi + hi*lo + lo*hi,
+// dropping lo*lo (relative 2^-22) and the TF32 truncation of lo (relative 2^-21).
 //
 // lud_tc_update: one 128 x 128 tile of C per CTA, 128 threads.  K is processed in chunks of KC:
 // all threads stage the chunk's A (128 x KC) and B^T (128 x KC) hi/lo parts, both as K-major
@@ -334,12 +332,7 @@ __device__ __forceinline__ void img_store4(float* __restrict__ img, int ng, int 
 // C -= A*B on 128 x 128 tiles: warp 0 lane 0 produces (bulk copies into an NS2-stage ring),
 // warp 1 lane 0 issues the 3xTF32 MMAs into TMEM and releases stages with tcgen05.commit; all
 // four warps run the epilogue (tcgen05.ld, C -= acc in place).
-// diag0 >= 0: the CTA whose tile starts at (diag0, diag0) also factors the 32 x 32 diagonal tile
-// of the next panel step (its warp 0 forms C - acc for that block in registers and runs
-// diag_factor instead of reducing it into C), which removes the separate lud_diag launch from
-// the factorisation's latency chain.
-__global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__ slot, int n, Args args, Img im,
-                                                      int diag0) {
+__global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__ slot, int n, Args args, Img im) {
     constexpr int PART = BM * KC2 * 4;
     constexpr int STAGE = 4 * PART;
     constexpr uint32_t SBO = KC2 * 32;
@@ -420,40 +413,6 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
 
     const int r = row0 + warp * 32 + lane;
     const int ncols = min(BN, cend - col0);
-    const bool dtile = diag0 >= 0 && row0 == diag0 && col0 == diag0;  // this CTA owns the next diagonal tile
-    if (dtile && warp == 0) {
-        uint32_t v[32];
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-              "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
-              "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
-              "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-            : "r"(tmem));
-        asm volatile("tcgen05.wait::ld.sync.aligned;"
-                     : "+r"(v[0]), "+r"(v[1]), "+r"(v[2]), "+r"(v[3]), "+r"(v[4]), "+r"(v[5]), "+r"(v[6]),
-                       "+r"(v[7]), "+r"(v[8]), "+r"(v[9]), "+r"(v[10]), "+r"(v[11]), "+r"(v[12]), "+r"(v[13]),
-                       "+r"(v[14]), "+r"(v[15]), "+r"(v[16]), "+r"(v[17]), "+r"(v[18]), "+r"(v[19]),
-                       "+r"(v[20]), "+r"(v[21]), "+r"(v[22]), "+r"(v[23]), "+r"(v[24]), "+r"(v[25]),
-                       "+r"(v[26]), "+r"(v[27]), "+r"(v[28]), "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
-                     :
-                     : "memory");
-        const int rd = min(32, n - diag0);
-        float a[32];
-        const float* crow = A + (size_t)(diag0 + lane) * n + diag0;
-#pragma unroll
-        for (int j = 0; j < 32; ++j)  // C - acc of the diagonal block, as the epilogue would store it
-            a[j] = (lane < rd && j < rd) ? __fsub_rn(crow[j], __uint_as_float(v[j])) : 0.f;
-        diag_factor<32>(a, rd, lane);
-        if (lane < rd) {
-            float* wrow = A + (size_t)(diag0 + lane) * n + diag0;
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-                if (j < rd) wrow[j] = a[j];
-        }
-    }
     if (vec && (ncols & 3) == 0) {
         // Epilogue through the L2: -acc rows staged in the (now idle) pipeline shared memory,
         // then one bulk reduce-add (cp.reduce.async.bulk .add.f32) per row into C.  x + (-y) is
@@ -489,16 +448,15 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
         }
         // generic-proxy writes -> async proxy (bulk copy engine) reads
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        const int skip = (dtile && warp == 0) ? 32 : 0;  // the diagonal block was stored factored
-        if (r < rend && ncols > skip)
+        if (r < rend)
             asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
-                             A + (size_t)r * n + col0 + skip),
-                         "r"(smem_u32(row_s + skip * 4)), "r"((ncols - skip) * 4)
+                             A + (size_t)r * n + col0),
+                         "r"(smem_u32(row_s)), "r"(ncols * 4)
                          : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     } else
-    for (int jb = (dtile && warp == 0) ? 1 : 0; jb < BN / 32; ++jb) {  // ragged or unaligned C: RMW per row
+    for (int jb = 0; jb < BN / 32; ++jb) {  // ragged or unaligned C: RMW per row
         uint32_t v[32];
         const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(jb * 32);
         asm volatile(
@@ -595,7 +553,7 @@ inline void launch_update2(float* const* slot, int n, const Rect* rs, int nr, in
     tc_split<<<dim3(grid_s, 2), 256, 0, s>>>(slot, n, img_a, img_b, base, k0, kk, ng, nchunks);
     Img im{img_a, img_b, base, base, ng, ng, 0};
     const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
-    lud_tc_update2<<<grid, 128, smem_bytes2(), s>>>(slot, n, a, im, -1);
+    lud_tc_update2<<<grid, 128, smem_bytes2(), s>>>(slot, n, a, im);
 }
 
 }  // namespace tc

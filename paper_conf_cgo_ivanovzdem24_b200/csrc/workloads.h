@@ -77,12 +77,22 @@ constexpr int NB = 128;                      // block size (the tensor-core upda
 size_t mimg_floats();                        // diagonal-block payload (U, L^T images, 1/u)
 int img_groups(int64_t rows);                // 8-row groups of an operand image for `rows`
 size_t img_floats(int64_t rows);             // floats of such an image (hi + lo, K = 128)
-rodinia_status diag(float* A, int lda, int r, float* mimg, cudaStream_t s);
-rodinia_status trsm(float* A, int lda, bool lower, int count, float* img, int ng, const float* mimg,
-                    cudaStream_t s);
+// The matrix pointer is read on the device from *slot (CUDA-graph reuse); off = element offset.
+// prio: cudaLaunchAttributePriority of the launch (0 = none; graph capture keeps it per node)
+rodinia_status diag(float* const* slot, size_t off, int lda, int r, float* mimg, cudaStream_t s, int prio = 0);
+struct TrsmJob {        // L rows (lower = 1: row t at A + t*lda) or U columns (column t at A + t),
+    float* const* slot;    // A = *slot + off
+    size_t off;
+    int lda, lower, count;
+    float* img;            // operand image (ng 8-row groups), image row = thread index
+    int ng;
+};
+rodinia_status trsm(const TrsmJob* job, int njobs, const float* mimg, cudaStream_t s, int prio = 0);  // one launch
 rodinia_status set_slot(float** slot, float* a, cudaStream_t s);
-rodinia_status update(float* const* slot, int lda, int r0, int m, int c0, int nn, const float* ia, int nga,
-                      const float* ib, int ngb, cudaStream_t s);
+// A -= L U over up to two rectangles rect[i] = {r0, m, c0, nn} of the local matrix; the operand
+// images start at local row a_base / column b_base (the trailing part's first row / column)
+rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr, int a_base, const float* ia,
+                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio = 0);
 }  // namespace ldist
 
 }  // namespace rg
