@@ -59,6 +59,16 @@ if want("lud"):
                      (16, (4, 1, 1, 2, 1, 1, STREAM)), (32, (2, 1, 1, 1, 1, 1, STREAM)), (128, None)]:
         a = A.clone()
         rg.rodinia_lud(a, panel, g=g)
+    B = torch.from_numpy(synth.lud_rodinia_matrix(301)).cuda()  # n % 4 != 0: scalar paths of panel 128
+    rg.rodinia_lud(B.clone(), 128)
+    # 2-D block-cyclic LU (LOCAL communicator): 2 x 2 on n = 300, 1 x 3 on n = 301
+    from paper_conf_cgo_ivanovzdem24_b200 import dist
+    for M, prow, pcol in [(A, 2, 2), (B, 1, 3)]:
+        parts = dist.block_cyclic_scatter(M, prow, pcol)
+        comm = dist.HaloComm.local_slabs(prow * pcol)
+        comm.lud(parts, M.shape[0], prow, pcol)
+        torch.cuda.synchronize()
+        comm.close()
     torch.cuda.synchronize()
     print("lud ok", flush=True)
 if want("hotspot3d"):
