@@ -279,6 +279,10 @@ __global__ void __launch_bounds__((P / TX) * (P / TY),
 // elements, A rows requested two rows ahead.  Per element the arithmetic is the same sequence as
 // every other variant (sum_i l_i u_i ascending with fma, then a -= sum), so results are
 // bit-identical for a fixed panel width.  Bound: HBM (8 B per element per step) at P = 16.
+#ifndef RG_LUD_RING
+#define RG_LUD_RING 8
+#endif
+constexpr int LUD_RING = RG_LUD_RING;  // rows in flight per thread (cp.async ring depth)
 template <int P, int V>
 __global__ void __launch_bounds__(256)
     lud_internal_stream(float* const* __restrict__ slot, int n, int k, int chunk_tiles, int unused) {
@@ -327,6 +331,59 @@ __global__ void __launch_bounds__(256)
             for (int v = 0; v < V; ++v) a[v] = cbase + v < n ? row[cbase + v] : 0.f;
         }
     };
+    if (vec) {
+        // A rows through a per-thread cp.async ring in shared memory (slots [LUD_RING][256][V],
+        // thread-private, no barrier): LUD_RING - 1 rows requested ahead of their use
+        float* ring = Lst + (((r1 - r0) * P + 3) & ~3);
+        const int nrows = r1 - r0;
+        auto issue = [&](int rr) {
+            if (rr < nrows) {
+                const float* src = A + (size_t)(r0 + rr) * n + cbase;
+                float* dst = ring + ((rr % LUD_RING) * 256 + threadIdx.x) * V;
+#pragma unroll
+                for (int q = 0; q < V / 4; ++q)
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(
+                                     (uint32_t)__cvta_generic_to_shared(dst + 4 * q)),
+                                 "l"(src + 4 * q));
+            }
+            asm volatile("cp.async.commit_group;\n" ::);
+        };
+#pragma unroll
+        for (int rr = 0; rr < LUD_RING - 1; ++rr) issue(rr);
+        for (int rr = 0; rr < nrows; ++rr) {
+            asm volatile("cp.async.wait_group %0;\n" ::"n"(LUD_RING - 2));  // row rr has landed
+            float a[V];
+            const float* slotp = ring + ((rr % LUD_RING) * 256 + threadIdx.x) * V;
+#pragma unroll
+            for (int q = 0; q < V / 4; ++q) {
+                const float4 t = reinterpret_cast<const float4*>(slotp)[q];
+                a[4 * q] = t.x; a[(4 * q + 1) % V] = t.y; a[(4 * q + 2) % V] = t.z; a[(4 * q + 3) % V] = t.w;
+            }
+            issue(rr + LUD_RING - 1);  // into the slot read one row ago
+            const float* l = Lst + rr * P;
+            float sum[V];
+#pragma unroll
+            for (int v = 0; v < V; ++v) sum[v] = 0.f;
+#pragma unroll
+            for (int i4 = 0; i4 < P / 4; ++i4) {
+                const float4 l4 = reinterpret_cast<const float4*>(l)[i4];
+                const float lv[4] = {l4.x, l4.y, l4.z, l4.w};
+#pragma unroll
+                for (int ii = 0; ii < 4; ++ii)
+#pragma unroll
+                    for (int v = 0; v < V; ++v) sum[v] = __fmaf_rn(lv[ii], u[4 * i4 + ii][v], sum[v]);
+            }
+            float* row = A + (size_t)(r0 + rr) * n + cbase;
+#pragma unroll
+            for (int q = 0; q < V / 4; ++q)
+                reinterpret_cast<float4*>(row)[q] =
+                    make_float4(__fsub_rn(a[4 * q], sum[4 * q]), __fsub_rn(a[(4 * q + 1) % V], sum[(4 * q + 1) % V]),
+                                __fsub_rn(a[(4 * q + 2) % V], sum[(4 * q + 2) % V]),
+                                __fsub_rn(a[(4 * q + 3) % V], sum[(4 * q + 3) % V]));
+        }
+        asm volatile("cp.async.wait_group 0;\n" ::);
+        return;
+    }
     float a0[V], a1[V];
     ld(r0, a0);
     if (r0 + 1 < r1) ld(r0 + 1, a1);
@@ -512,7 +569,8 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
         pl->v = nullptr;
         pl->bx = 1;
         pl->by = g.block_y;  // rows per CTA in 16-row tiles
-        pl->smem = (size_t)16 * g.block_y * panel * sizeof(float);
+        // L21 rows of the chunk + the cp.async ring (LUD_RING rows x 256 threads x V)
+        pl->smem = (size_t)16 * g.block_y * panel * sizeof(float) + (size_t)LUD_RING * 256 * g.thread_x * sizeof(float);
         if (pl->smem > 227 * 1024) return set_error(RODINIA_E_SMEM, "lud: stream chunk needs %zu B shared memory", pl->smem);
         return boundary_filter(RODINIA_LUD, pl->sv->key, 256, (int)pl->smem, g.flags);
     }
