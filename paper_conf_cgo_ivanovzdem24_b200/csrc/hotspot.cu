@@ -231,7 +231,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
                                                const float* __restrict__ tin, const float* __restrict__ pw,
                                                float* __restrict__ tout, int s, int ystart, int R, int C, int ylo,
                                                int yhi, int sc0, int col0, const HsCoef& cf,
-                                               const float*& tsrc, const float*& psrc) {
+                                               const float*& tsrc, const float*& psrc, float*& optr) {
     constexpr int S0 = K % 3, S1 = (K + 1) % 3, S2 = (K + 2) % 3;
     constexpr int DP = HsRing<H>::DP;
     const int g0 = ystart + s;
@@ -291,7 +291,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
         } else if (g >= ylo && g < yhi) {
             // level H: write the lane's cells that lie in the band's output columns
             constexpr int s_lo = H, s_hi = 32 * V - H;  // staged-column range of the output
-            float* orow = tout + (size_t)g * C + col0;
+            float* orow = optr;  // = tout + g * C + col0 (running pointer: no per-step 64-bit multiply)
             if constexpr (!EC && (H % V == 0) && V <= 4) {
                 if (sc0 >= s_lo && sc0 < s_hi) {
                     typename VecT<V>::T t;
@@ -316,6 +316,7 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
             }
         }
     }
+    optr += C;
 }
 
 template <int V, int H, bool EC, bool ER>
@@ -336,23 +337,25 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
     // fast-path source pointers (only dereferenced when !EC && !ER: all requested rows exist)
     const float* tsrc = tin + (size_t)max(ystart, 0) * C + col0;
     const float* psrc = pw + (size_t)max(ystart - 1, 0) * C + col0;
+    // output row of level H at step s: ystart + s - H (only dereferenced inside [y0, y1))
+    float* optr = tout + (ptrdiff_t)(ystart - H) * C + col0;
 #pragma unroll
     for (int k = 0; k < HS_DT - 1; ++k)
         hs_issue_step<V, H, EC, ER>(tring, pring, tin, pw, k, ystart, R, C, col0, sc0, tsrc, psrc);
     int s = 0;
     // prologue: the top-halo trapezoid (levels switched on two steps apart)
     for (; RG_HS_TRAP && s + 3 <= nsteps && s < 2 * H; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 2, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
+        hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
+        hs_stream_step<V, H, 2, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
     }
     for (; s + 3 <= nsteps; s += 3) {
-        hs_stream_step<V, H, 0, EC, ER, false>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 1, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-        hs_stream_step<V, H, 2, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+        hs_stream_step<V, H, 0, EC, ER, false>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
+        hs_stream_step<V, H, 1, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
+        hs_stream_step<V, H, 2, EC, ER, false>(ring, tring, pring, tin, pw, tout, s + 2, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
     }
-    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
-    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc);
+    if (s < nsteps) hs_stream_step<V, H, 0, EC, ER, true>(ring, tring, pring, tin, pw, tout, s, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
+    if (s + 1 < nsteps) hs_stream_step<V, H, 1, EC, ER, true>(ring, tring, pring, tin, pw, tout, s + 1, ystart, R, C, y0, y1, sc0, col0, cf, tsrc, psrc, optr);
     asm volatile("cp.async.wait_group 0;\n" ::);  // drain before the rings are reused
 }
 

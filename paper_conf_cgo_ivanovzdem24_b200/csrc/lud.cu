@@ -773,7 +773,7 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
         if ((is_stream ? lud::kStreamInt[vi - ni].p : lud::kInternal[vi].p) != panel) continue;
         for (int bx : {1, 2, 4, 7})
             for (int by : {1, 2, 4, 8, 16}) {
-                if (is_stream ? (bx != 1 || by < 4) : by > 4) continue;
+                if (is_stream ? (bx != 1 || by > 8) : by > 4) continue;  // stream: 16..128-row chunks
                 rodinia_tune_row row;
                 memset(&row, 0, sizeof row);
                 row.g = g0;
