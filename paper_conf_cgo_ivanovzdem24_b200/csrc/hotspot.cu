@@ -288,7 +288,9 @@ __device__ __forceinline__ void hs_stream_step(float (&ring)[H][3][V], float* tr
         if (l + 1 < H) {
 #pragma unroll
             for (int v = 0; v < V; ++v) ring[l + 1 < H ? l + 1 : 0][S2][v] = res[v];
-        } else if (g >= ylo && g < yhi) {
+        } else if ((!PRO && RG_HS_TRAP) || (g >= ylo && g < yhi)) {
+            // (the steady loop runs steps 2H <= s <= nsteps - 1 only, whose level-H rows
+            // y0 - 2H + s all lie in [y0, y1): no row test there)
             // level H: write the lane's cells that lie in the band's output columns
             constexpr int s_lo = H, s_hi = 32 * V - H;  // staged-column range of the output
             float* orow = optr;  // = tout + g * C + col0 (running pointer: no per-step 64-bit multiply)
