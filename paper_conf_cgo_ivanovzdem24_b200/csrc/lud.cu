@@ -856,7 +856,12 @@ constexpr int D128_LT = 132;                   // transposed L sub-panel: LT[k][
 #define LUD_PROBE(i)
 #define LUD_PROBE_W(i)
 #endif
-constexpr int D128_IMG = 128 * D128_LD;        // one 128 x 128 image padded to D128_LD
+// The payload lud_trsm128 reads: U11 and L11^T in a block-upper packed layout (row k of block
+// b = k/32 keeps columns [32b, 128): the only ones a solve reads), then RN(1/u_jj).
+constexpr int D128_IMG = 32 * (128 + 96 + 64 + 32);  // 10240 floats per packed image
+__host__ __device__ constexpr int bup_row(int k) {    // offset of row k's first stored column
+    return 4096 * (k >> 5) - 512 * (k >> 5) * ((k >> 5) - 1) + (k & 31) * (128 - 32 * (k >> 5));
+}
 constexpr size_t d128_mimg_floats() { return (size_t)2 * D128_IMG + 128; }
 
 // RN(a / b) from rb = RN(1 / b) (Markstein): q0 = RN(a rb) lies within one ulp of a/b, the
@@ -1080,11 +1085,13 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     // image built in shared memory meanwhile
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncthreads();
-    if (tid == 0) {
-        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg),
-                     "r"(tc::smem_u32(S)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
+    if (tid == 0)
         asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + 2 * D128_IMG),
                      "r"(tc::smem_u32(rinv)), "r"(512u) : "memory");
+    if (tid >= 128) {  // packed U image: row k, columns [32b, 128)
+        const int k = tid - 128, b = k >> 5;
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + bup_row(k)),
+                     "r"(tc::smem_u32(S + k * LD + 32 * b)), "r"((uint32_t)((128 - 32 * b) * 4)) : "memory");
     }
     if (bulk) {
         if (tid < 128)
@@ -1104,9 +1111,10 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     for (int e = tid; e < 128 * PADC; e += 256) T[(e / PADC) * LD + 128 + (e % PADC)] = 0.f;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncthreads();
-    if (tid == 0) {
-        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + D128_IMG),
-                     "r"(tc::smem_u32(T)), "r"((uint32_t)(D128_IMG * 4)) : "memory");
+    if (tid < 128) {  // packed L^T image
+        const int k = tid, b = k >> 5;
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(mimg + D128_IMG + bup_row(k)),
+                     "r"(tc::smem_u32(T + k * LD + 32 * b)), "r"((uint32_t)((128 - 32 * b) * 4)) : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
     }
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // shared memory read before exit
@@ -1133,7 +1141,7 @@ constexpr size_t d128_smem() { return ((size_t)(132 + 128) * D128_LD + 32 * D128
 // Each solved piece is written to A and, split hi/lo, to the tensor-core operand image `img`
 // (ng 8-row groups) of the update, image row = thread index.
 constexpr int TR_T = 64, TR_RLD = 129;
-constexpr size_t trsm_smem() { return ((size_t)D128_IMG + 128 + (size_t)TR_T * TR_RLD) * sizeof(float); }
+constexpr size_t trsm_smem() { return ((size_t)D128_IMG + 128 + (size_t)TR_T * TR_RLD) * sizeof(float); }  // 74.5 KB: 3 CTAs/SM
 
 __device__ __forceinline__ void trsm_load(const float* A, int lda, bool lower, bool vec, bool own, int idx, int c0,
                                           float2 (&x)[16]) {
@@ -1195,16 +1203,21 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
 #pragma unroll 1
     for (int p = 0; p < 128; p += 32) {
         if (p + 32 < 128) trsm_load(A, lda, lower, vec, own, idx, p + 32, xn);
+        for (int b = 0; b < p / 32; ++b) {  // the rows of earlier blocks: columns p.. of row k
+            const float* mb = M + bup_row(32 * b) + (p - 32 * b);
+            const int lb = 128 - 32 * b;
+            const float* rb = Rt + 32 * b;
 #pragma unroll 4
-        for (int k = 0; k < p; ++k) {
-            const float nl = -Rt[k];
-            const float2 nl2 = make_float2(nl, nl);
-            const float4* mr = reinterpret_cast<const float4*>(M + k * LD + p);
+            for (int kk = 0; kk < 32; ++kk) {
+                const float nl = -rb[kk];
+                const float2 nl2 = make_float2(nl, nl);
+                const float4* mr = reinterpret_cast<const float4*>(mb + kk * lb);
 #pragma unroll
-            for (int q = 0; q < 8; ++q) {
-                const float4 m = mr[q];
-                x[2 * q] = __ffma2_rn(nl2, make_float2(m.x, m.y), x[2 * q]);
-                x[2 * q + 1] = __ffma2_rn(nl2, make_float2(m.z, m.w), x[2 * q + 1]);
+                for (int q = 0; q < 8; ++q) {
+                    const float4 m = mr[q];
+                    x[2 * q] = __ffma2_rn(nl2, make_float2(m.x, m.y), x[2 * q]);
+                    x[2 * q + 1] = __ffma2_rn(nl2, make_float2(m.z, m.w), x[2 * q + 1]);
+                }
             }
         }
         float xs[32];
@@ -1212,7 +1225,7 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
         for (int q = 0; q < 16; ++q) { xs[2 * q] = x[q].x; xs[2 * q + 1] = x[q].y; }
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
-            const float4* mr = reinterpret_cast<const float4*>(M + (p + j) * LD + p);
+            const float4* mr = reinterpret_cast<const float4*>(M + bup_row(p + j));  // columns p..
             float mv[32];
 #pragma unroll
             for (int q = j / 4; q < 8; ++q) {
