@@ -217,8 +217,10 @@ rodinia_status rodinia_pathfinder_host(const int32_t* wall, int64_t rows, int64_
  * lud -- Rodinia lud (blocked Doolittle LU, no pivoting), L1-L6.  a (n x n fp32)
  * is factored in place: unit-diagonal L strictly below the diagonal, U on and above.
  * panel: block (panel) width; 16 = Rodinia's BLOCK_SIZE (0 => 16).  Supported: 16, 32, and
- * 128 = two-level blocking (inner panel 32) whose rank-128 trailing updates run on the tensor
- * cores (tcgen05.mma kind::tf32 with the 3xTF32 split; g is ignored there).
+ * 128: per 128-wide block column the diagonal block is factored by one CTA, L21 / U12 are solved
+ * one thread per row / column, and the rank-128 trailing update runs on the tensor cores
+ * (tcgen05.mma kind::tf32 with the 3xTF32 split; g is ignored there); its
+ * quotients are IEEE quotients formed from the pivot's correctly rounded reciprocal.
  * The panel width changes fp32 rounding order and is reported separately from coarsening
  * (reading L5).  Zero pivots give inf/NaN (no pivoting, as Rodinia). */
 rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
