@@ -2,8 +2,9 @@
 //
 // Operation: Doolittle LU without pivoting, packed in place (DESIGN.md §3 L1-L6), computed
 // with Rodinia's blocked structure.  For panel step k (offset o = P*k):
-//   lud_diag      in-tile Doolittle of the P x P diagonal tile (one CTA);
-//   lud_perim     U12 = L11^-1 A12 (unit-lower forward substitution) for every tile right of
+//   lud_perim     in-tile Doolittle of the P x P diagonal tile (Rodinia's lud_diagonal, done by
+//                 warp 0 of every CTA, so no separate launch sits on the chain), then
+//                 U12 = L11^-1 A12 (unit-lower forward substitution) for every tile right of
 //                 the diagonal, L21 = A21 U11^-1 for every tile below it;
 //   lud_internal  A22 -= L21 * U12 for every trailing tile (the paper's "main lud kernel",
 //                 PAPER.md:315-353, which its coarsening study targets).
@@ -15,7 +16,8 @@
 // accumulation order (sum over i ascending, then a -= sum) is the same in every variant, so
 // for a fixed panel width every (t, b) variant is bit-identical (reading L5).
 //
-// The 3*ceil(n/P)-2 launches of one factorisation are captured once into a CUDA graph per
+// lud_diag_final writes the factored diagonal tiles back at the end (and factors the last one).
+// The 2*ceil(n/P)-1 launches of one factorisation are captured once into a CUDA graph per
 // (device, n, P, granularity) and replayed; kernels read the matrix pointer from a device slot
 // the call sets first, so one graph serves every matrix of that size.
 #include <cuda_runtime.h>
@@ -34,25 +36,6 @@
 
 namespace rg {
 
-// ------------------------------------------------------------------ diagonal tile
-// One warp.  Lane i holds row i of the tile in registers; step k broadcasts row k with warp
-// shuffles and every lane below it subtracts l_ik * u_kj.  Per element this is exactly
-// Doolittle's sequence (products subtracted in ascending k, L divided by the pivot after its
-// k < j terms), computed with separate multiply and subtract as in Rodinia's lud_diagonal.
-template <int P>
-__global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, int n, int k) {
-    float* A = *slot;
-    const int o = k * P, r = min(P, n - o), lane = threadIdx.x;
-    float a[P];
-    const bool own = lane < r;
-#pragma unroll
-    for (int j = 0; j < P; ++j) a[j] = (own && j < r) ? A[(size_t)(o + lane) * n + o + j] : 0.f;
-    tc::diag_factor<P>(a, r, lane);
-#pragma unroll
-    for (int j = 0; j < P; ++j)
-        if (own && j < r) A[(size_t)(o + lane) * n + o + j] = a[j];
-}
-
 // ------------------------------------------------------------------ perimeter tiles
 // CTA j handles the j-th tile right of the diagonal and the j-th tile below it: lanes 0..P-1
 // each own one column of U12 = L11^-1 A12 (forward substitution, unit-lower L11), lanes
@@ -64,8 +47,13 @@ __global__ void __launch_bounds__(32) lud_diag(float* const* __restrict__ slot, 
 // time with 128-bit shared loads; per element the subtractions run in ascending j exactly as in
 // the two separate loops this replaces (same bits), with half the code (the fully unrolled pair
 // of solves overflowed the instruction cache: "no instruction" was the top stall, ncu r02f).
+// The diagonal tile of step k (full: only the last tile can be partial, and it has no
+// perimeter) is factored by warp 0 of every perimeter CTA itself (diag_factor, the lud_diag
+// sequence: same bits), so no separate diagonal launch sits on the chain; A keeps the unfactored
+// tile until the end of the factorisation (no later kernel reads it), CTA 0 stores the factored
+// tile in dscr[k], and lud_diag_final writes all of them into A (and factors the last tile).
 template <int P>
-__device__ __forceinline__ void lud_perim_body(float* A, int n, int k) {
+__device__ __forceinline__ void lud_perim_body(float* A, int n, int k, float* __restrict__ dscr) {
     constexpr int LD = P + 4;  // 16-byte aligned rows
     __shared__ __align__(16) float msm[2][P][LD];  // [0]: L11 = dia (row-major), [1]: U11^T
     __shared__ float tile[2][P][P + 1];            // [0]: row tile A12, [1]: column tile A21
@@ -73,14 +61,29 @@ __device__ __forceinline__ void lud_perim_body(float* A, int n, int k) {
     const int tb = o + P * (blockIdx.x + 1);  // first row/col of this perimeter tile
     const int w = min(P, n - tb);             // its width (last tile may be partial)
     const int tx = threadIdx.x;
-    // fully unrolled: all 3P/2 loads of a thread are in flight at once (one memory round trip;
+    if (tx < 32) {
+        float a[P];
+        const bool own = tx < P;
+#pragma unroll
+        for (int j = 0; j < P; ++j) a[j] = own ? A[(size_t)(o + tx) * n + o + j] : 0.f;
+        tc::diag_factor<P>(a, P, tx);
+        if (own) {
+#pragma unroll
+            for (int j = 0; j < P; ++j) {
+                msm[0][tx][j] = a[j];
+                msm[1][j][tx] = a[j];
+            }
+            if (blockIdx.x == 0) {
+#pragma unroll
+                for (int j = 0; j < P; ++j) dscr[((size_t)k * P + tx) * P + j] = a[j];
+            }
+        }
+    }
+    // fully unrolled: all P loads of a thread are in flight at once (one memory round trip;
     // the rolled loop cost one round trip per iteration, ~16 us per launch at P = 32)
 #pragma unroll
     for (int e0 = 0; e0 < P * P; e0 += 2 * P) {
         const int e = e0 + tx, i = e / P, j = e % P;
-        const float d = A[(size_t)(o + i) * n + o + j];
-        msm[0][i][j] = d;
-        msm[1][j][i] = d;
         tile[0][i][j] = j < w ? A[(size_t)(o + i) * n + tb + j] : 0.f;
         tile[1][i][j] = i < w ? A[(size_t)(tb + i) * n + o + j] : 0.f;
     }
@@ -114,8 +117,32 @@ __device__ __forceinline__ void lud_perim_body(float* A, int n, int k) {
 }
 
 template <int P>
-__global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k) {
-    lud_perim_body<P>(*slot, n, k);
+__global__ void __launch_bounds__(2 * P) lud_perim(float* const* __restrict__ slot, int n, int k, float* dscr) {
+    lud_perim_body<P>(*slot, n, k, dscr);
+}
+
+// End of a panel-16/32 factorisation: CTA k < m-1 writes the factored diagonal tile k (dscr)
+// into A; CTA m-1 factors the last diagonal tile in A (after the last trailing update).
+template <int P>
+__global__ void __launch_bounds__(32) lud_diag_final(float* const* __restrict__ slot, int n, const float* __restrict__ dscr) {
+    float* A = *slot;
+    const int m = (n + P - 1) / P, k = blockIdx.x, o = k * P, lane = threadIdx.x;
+    if (k < m - 1) {
+        if (lane < P) {
+#pragma unroll
+            for (int j = 0; j < P; ++j) A[(size_t)(o + lane) * n + o + j] = dscr[((size_t)k * P + lane) * P + j];
+        }
+        return;
+    }
+    const int r = min(P, n - o);
+    float a[P];
+    const bool own = lane < r;
+#pragma unroll
+    for (int j = 0; j < P; ++j) a[j] = (own && j < r) ? A[(size_t)(o + lane) * n + o + j] : 0.f;
+    tc::diag_factor<P>(a, r, lane);
+#pragma unroll
+    for (int j = 0; j < P; ++j)
+        if (own && j < r) A[(size_t)(o + lane) * n + o + j] = a[j];
 }
 
 
@@ -500,7 +527,6 @@ __global__ void lud_set_slot(float** slot, float* a) { *slot = a; }
 namespace lud {
 
 typedef void (*IntFn)(float* const*, int, int, int, int);
-typedef void (*DPFn)(float* const*, int, int);
 struct Variant { int p, tx, ty, mode; IntFn fn; const char* key; };
 
 #define RG_LI(P, TX, TY, M) {P, TX, TY, M, lud_internal<P, TX, TY, M>, "void rg::lud_internal<" #P ", " #TX ", " #TY ", " #M ">"}
@@ -589,14 +615,14 @@ rodinia_status plan(const rodinia_granularity& g, int panel, Plan* pl) {
                            g.flags);  // compile-time filter at the boundary
 }
 
-static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
+typedef void (*PerimFn)(float* const*, int, int, float*);
+typedef void (*DiagFinalFn)(float* const*, int, const float*);
+static int launch_all(const Plan& pl, float** slot, int n, float* dscr, cudaStream_t s) {
     const int P = pl.p, m = (n + P - 1) / P;
-    DPFn diag = P == 16 ? (DPFn)lud_diag<16> : (DPFn)lud_diag<32>;
-    DPFn perim = P == 16 ? (DPFn)lud_perim<16> : (DPFn)lud_perim<32>;
-    for (int k = 0; k < m; ++k) {
-        diag<<<1, 32, 0, s>>>(slot, n, k);
-        if (k == m - 1) break;
-        perim<<<m - k - 1, 2 * P, 0, s>>>(slot, n, k);
+    PerimFn perim = P == 16 ? (PerimFn)lud_perim<16> : (PerimFn)lud_perim<32>;
+    DiagFinalFn fin = P == 16 ? (DiagFinalFn)lud_diag_final<16> : (DiagFinalFn)lud_diag_final<32>;
+    for (int k = 0; k + 1 < m; ++k) {
+        perim<<<m - k - 1, 2 * P, 0, s>>>(slot, n, k, dscr);  // + the diagonal tile of step k
         const int rem = m - k - 1;
         if (pl.sv) {
             const int width = n - P * (k + 1);
@@ -608,6 +634,8 @@ static void launch_all(const Plan& pl, float** slot, int n, cudaStream_t s) {
         dim3 block(P / pl.v->tx, P / pl.v->ty);
         pl.v->fn<<<grid, block, pl.smem, s>>>(slot, n, k, pl.bx, pl.by);
     }
+    fin<<<m, 32, 0, s>>>(slot, n, dscr);
+    return 2 * (m - 1) + 1;
 }
 
 // One captured factorisation per (device, n, plan).  The matrix pointer reaches the kernels
@@ -623,6 +651,7 @@ struct GraphEntry {
     cudaKernelNodeParams rootp = {};
     float** slot = nullptr;
     float* img = nullptr;   // panel-128 path: the two tensor-core operand images
+    float* dscr = nullptr;  // panel 16/32: the factored diagonal tiles (written back at the end)
     int launches = 0;
 };
 static std::mutex g_mu;
@@ -644,6 +673,7 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         const size_t fimg = std::max(tc::img_floats(n), ldist::img_floats(n));
         if (pl.tc && !ge.img)  // 4 operand images + the diagonal-block payload (v3)
             RG_CUDA(cudaMalloc(&ge.img, (4 * fimg + ldist::mimg_floats()) * sizeof(float)));
+        if (!pl.tc && !ge.dscr) RG_CUDA(cudaMalloc(&ge.dscr, (size_t)m * pl.p * pl.p * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
         cudaStream_t cs, cs2;
@@ -664,7 +694,7 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
             float* const imgs[4] = {ge.img, ge.img + f, ge.img + 2 * f, ge.img + 3 * f};
             nl = tc::launch_all3(ge.slot, n, imgs, ge.img + 4 * f, cs, cs2, ev[0], ev[1], ev[2], prio_hi);
         } else {
-            launch_all(pl, ge.slot, n, cs);
+            nl = launch_all(pl, ge.slot, n, ge.dscr, cs);
         }
         cudaError_t e = cudaStreamEndCapture(cs, &graph);
         cudaStreamDestroy(cs);
