@@ -1294,7 +1294,9 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
 
 namespace ldist {
 size_t mimg_floats() { return d128_mimg_floats(); }
-int img_groups(int64_t rows) { return (int)(((rows + 127) / 128 + 1) * 16); }
+// padded to whole 256-wide tiles plus one spare (the update's 128 x 256 tiles read B columns
+// up to the next multiple of 256 past the rectangle's start)
+int img_groups(int64_t rows) { return (int)(((rows + 255) / 256 + 1) * 32); }
 size_t img_floats(int64_t rows) { return (size_t)16 * img_groups(rows) * tc::KC2 * 8; }
 
 rodinia_status diag(float* const* slot, size_t off, int lda, int r, float* mimg, cudaStream_t s, int prio) {
@@ -1342,20 +1344,35 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
                       int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio) {
     static bool attr = false;
     if (!attr) {
-        RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update2, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)tc::smem_bytes2()));
+        RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)tc::Upd3<128>::smem()));
+        RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<256>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)tc::Upd3<256>::smem()));
         attr = true;
     }
+    // 128 x 256 C tiles when every rectangle is wider than 128 columns (the remainder update),
+    // else 128 x 128 (block column k+1 is exactly 128 wide)
+    bool wide = true;
+    int live = 0;
+    for (int i = 0; i < nr && i < 2; ++i)
+        if (rect[i][1] > 0 && rect[i][3] > 0) {
+            ++live;
+            wide = wide && rect[i][3] > 128;
+        }
+    if (live == 0) return RODINIA_OK;
+    const int bn = wide ? 256 : 128;
     tc::Args a;
     a.nrect = 0;
     for (int i = 0; i < nr && i < 2; ++i)  // rect[i] = {r0, m, c0, nn}
         if (rect[i][1] > 0 && rect[i][3] > 0)
-            a.rect[a.nrect++] = tc::make_rect(rect[i][0], rect[i][2], rect[i][1], rect[i][3], 0, LD_NB);
-    if (a.nrect == 0) return RODINIA_OK;
+            a.rect[a.nrect++] = tc::make_rect(rect[i][0], rect[i][2], rect[i][1], rect[i][3], 0, LD_NB, bn);
     if (a.nrect == 1) a.rect[1] = a.rect[0];
     const tc::Img im{ia, ib, a_base, b_base, nga, ngb, 0};
     const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
-    tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update2, dim3(grid), dim3(128), tc::smem_bytes2(), slot, lda, a, im);
+    if (wide)
+        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);
+    else
+        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<128>, dim3(grid), dim3(128), tc::Upd3<128>::smem(), slot, lda, a, im);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;

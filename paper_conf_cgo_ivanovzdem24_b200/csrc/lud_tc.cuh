@@ -504,6 +504,212 @@ __global__ void __launch_bounds__(128) lud_tc_update2(float* const* __restrict__
 
 constexpr size_t smem_bytes2() { return (size_t)NS2 * 4 * BM * KC2 * 4 + 128; }
 
+// v3 (round 2): the update with a BNT-wide C tile (128 or 256 columns; M = 128, accumulator
+// 128 lanes x BNT TMEM columns).  A 128 x 256 tile reads the same A panel once for twice the
+// outputs (the per-tile re-reads of the hi/lo panels from L2 are what bounded the 128 x 128
+// version on large trailing matrices); stages hold A hi/lo + B hi/lo of one 16-deep K chunk
+// (3 stages at 128 columns, 2 at 256: 96 KB, 2 CTAs and 2 x BNT <= 512 TMEM columns per SM).
+template <int BNT>
+struct Upd3 {
+    static constexpr int NS = BNT == 128 ? 3 : 2;
+    static constexpr int PA = BM * KC2 * 4;
+    static constexpr int PB = BNT * KC2 * 4;
+    static constexpr int STAGE = 2 * PA + 2 * PB;
+    static constexpr size_t smem() { return (size_t)NS * STAGE + 128; }
+    // kind::tf32, D f32, A and B K-major, M = 128, N = BNT
+    static constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BNT >> 3) << 17) |
+                                      ((uint32_t)(BM >> 4) << 24);
+};
+__device__ __forceinline__ void mma_tf32_i(uint32_t tmem, uint64_t ad, uint64_t bd, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem),
+        "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+}
+
+template <int BNT>
+__global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__ slot, int n, Args args, Img im) {
+    constexpr int NS = Upd3<BNT>::NS;
+    constexpr int PART = Upd3<BNT>::PA;   // one A part (hi or lo): 128 rows x KC2
+    constexpr int PARTB = Upd3<BNT>::PB;  // one B part: BNT columns x KC2
+    constexpr int STAGE = Upd3<BNT>::STAGE;
+    constexpr uint32_t SBO = KC2 * 32;
+    extern __shared__ __align__(1024) uint8_t sm[];
+    uint64_t* full = reinterpret_cast<uint64_t*>(sm + NS * STAGE);
+    uint64_t* empty = full + NS;
+    uint64_t* done = empty + NS;
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(done + 1);
+    float* A = *slot;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+
+    int b = blockIdx.x, ri = 0;
+    if (args.nrect == 2 && b >= args.rect[0].tiles) { b -= args.rect[0].tiles; ri = 1; }
+    const Rect rc = ri ? args.rect[1] : args.rect[0];
+    const int ty = b / rc.tiles_x, tx = b - ty * rc.tiles_x;
+    const int row0 = rc.r0 + ty * BM, col0 = rc.c0 + tx * BNT;
+    const int rend = rc.r0 + rc.m, cend = rc.c0 + rc.nn;
+    const bool vec = (n & 3) == 0;
+    const int nchunks = (rc.kk + KC2 - 1) / KC2;
+    const int ga = (row0 - im.a_base) >> 3, gb = (col0 - im.b_base) >> 3;
+
+    if (tid == 0) {
+        for (int i = 0; i < NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+        mbar_init(done, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)), "n"(BNT));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tslot;
+
+    if (tid == 0) {  // producer
+        for (int c = 0; c < nchunks; ++c) {
+            const int s = c % NS;
+            if (c >= NS) mbar_wait(&empty[s], ((c / NS) - 1) & 1);
+            uint8_t* st = sm + s * STAGE;
+            mbar_expect_tx(&full[s], STAGE);
+            const int ci = c + im.c0;
+            const float* ah = im.a + ((size_t)(ci * 2) * im.nga + ga) * (KC2 * 8);
+            const float* al = im.a + ((size_t)(ci * 2 + 1) * im.nga + ga) * (KC2 * 8);
+            const float* bh = im.b + ((size_t)(ci * 2) * im.ngb + gb) * (KC2 * 8);
+            const float* bl = im.b + ((size_t)(ci * 2 + 1) * im.ngb + gb) * (KC2 * 8);
+            bulk_g2s(st, ah, PART, &full[s]);
+            bulk_g2s(st + PART, al, PART, &full[s]);
+            bulk_g2s(st + 2 * PART, bh, PARTB, &full[s]);
+            bulk_g2s(st + 2 * PART + PARTB, bl, PARTB, &full[s]);
+        }
+    } else if (tid == 32) {  // MMA issuer
+        for (int c = 0; c < nchunks; ++c) {
+            const int s = c % NS;
+            mbar_wait(&full[s], (c / NS) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const uint32_t a_hi = smem_u32(sm + s * STAGE), a_lo = a_hi + PART, b_hi = a_hi + 2 * PART,
+                           b_lo = b_hi + PARTB;
+#pragma unroll
+            for (int ks = 0; ks < KC2 / 8; ++ks) {
+                const uint64_t adh = sm_desc(a_hi + ks * 256, 128, SBO), adl = sm_desc(a_lo + ks * 256, 128, SBO);
+                const uint64_t bdh = sm_desc(b_hi + ks * 256, 128, SBO), bdl = sm_desc(b_lo + ks * 256, 128, SBO);
+                mma_tf32_i(tmem, adl, bdh, Upd3<BNT>::idesc, (c | ks) != 0);
+                mma_tf32_i(tmem, adh, bdl, Upd3<BNT>::idesc, 1);
+                mma_tf32_i(tmem, adh, bdh, Upd3<BNT>::idesc, 1);
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                             smem_u32(&empty[s]))
+                         : "memory");
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                         smem_u32(done))
+                     : "memory");
+    }
+    __syncwarp();
+    mbar_wait(done, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+
+    const int r = row0 + warp * 32 + lane;
+    const int ncols = min(BNT, cend - col0);
+    if (vec && (ncols & 3) == 0) {
+        // Epilogue through the L2, 128 columns at a time: -acc rows staged in the (now idle)
+        // pipeline shared memory, then one bulk reduce-add (cp.reduce.async.bulk .add.f32) per
+        // row into C.  x + (-y) is x - y bit for bit, each element is added exactly once, and
+        // the SMs never read C.
+        constexpr int PITCH = 128 * 4 + 16;  // 528 B: conflict-free 16-byte row-per-lane stores
+        uint8_t* row_s = sm + (warp * 32 + lane) * PITCH;
+#pragma unroll 1
+        for (int h = 0; h < BNT / 128; ++h) {
+            const int nh = min(128, ncols - 128 * h);
+            if (nh <= 0) break;  // CTA-uniform
+            if (h > 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // row_s is free again
+#pragma unroll 1
+            for (int jb = 0; jb < 4; ++jb) {
+                uint32_t v[32];
+                const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(128 * h + jb * 32);
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                    "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                      "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+                      "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+                      "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+                    : "r"(taddr));
+                asm volatile("tcgen05.wait::ld.sync.aligned;"
+                             : "+r"(v[0]), "+r"(v[1]), "+r"(v[2]), "+r"(v[3]), "+r"(v[4]), "+r"(v[5]), "+r"(v[6]),
+                               "+r"(v[7]), "+r"(v[8]), "+r"(v[9]), "+r"(v[10]), "+r"(v[11]), "+r"(v[12]), "+r"(v[13]),
+                               "+r"(v[14]), "+r"(v[15]), "+r"(v[16]), "+r"(v[17]), "+r"(v[18]), "+r"(v[19]),
+                               "+r"(v[20]), "+r"(v[21]), "+r"(v[22]), "+r"(v[23]), "+r"(v[24]), "+r"(v[25]),
+                               "+r"(v[26]), "+r"(v[27]), "+r"(v[28]), "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
+                             :
+                             : "memory");
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                    *reinterpret_cast<float4*>(row_s + jb * 128 + q * 16) =
+                        make_float4(-__uint_as_float(v[4 * q]), -__uint_as_float(v[4 * q + 1]),
+                                    -__uint_as_float(v[4 * q + 2]), -__uint_as_float(v[4 * q + 3]));
+            }
+            // generic-proxy writes -> async proxy (bulk copy engine) reads
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            if (r < rend)
+                asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
+                                 A + (size_t)r * n + col0 + 128 * h),
+                             "r"(smem_u32(row_s)), "r"(nh * 4)
+                             : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    } else
+    for (int jb = 0; jb < BNT / 32; ++jb) {  // ragged or unaligned C: RMW per row
+        uint32_t v[32];
+        const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(jb * 32);
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+              "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+              "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+              "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+            : "r"(taddr));
+        asm volatile("tcgen05.wait::ld.sync.aligned;"
+                     : "+r"(v[0]), "+r"(v[1]), "+r"(v[2]), "+r"(v[3]), "+r"(v[4]), "+r"(v[5]), "+r"(v[6]),
+                       "+r"(v[7]), "+r"(v[8]), "+r"(v[9]), "+r"(v[10]), "+r"(v[11]), "+r"(v[12]), "+r"(v[13]),
+                       "+r"(v[14]), "+r"(v[15]), "+r"(v[16]), "+r"(v[17]), "+r"(v[18]), "+r"(v[19]),
+                       "+r"(v[20]), "+r"(v[21]), "+r"(v[22]), "+r"(v[23]), "+r"(v[24]), "+r"(v[25]),
+                       "+r"(v[26]), "+r"(v[27]), "+r"(v[28]), "+r"(v[29]), "+r"(v[30]), "+r"(v[31])
+                     :
+                     : "memory");
+        if (r < rend) {
+            float* crow = A + (size_t)r * n;
+            const int cb = col0 + jb * 32;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const int cc = cb + 4 * q;
+                if (vec && cc + 4 <= cend) {
+                    float4 t = *reinterpret_cast<float4*>(crow + cc);
+                    t.x = __fsub_rn(t.x, __uint_as_float(v[4 * q]));
+                    t.y = __fsub_rn(t.y, __uint_as_float(v[4 * q + 1]));
+                    t.z = __fsub_rn(t.z, __uint_as_float(v[4 * q + 2]));
+                    t.w = __fsub_rn(t.w, __uint_as_float(v[4 * q + 3]));
+                    *reinterpret_cast<float4*>(crow + cc) = t;
+                } else {
+#pragma unroll
+                    for (int e = 0; e < 4; ++e)
+                        if (cc + e < cend) crow[cc + e] = __fsub_rn(crow[cc + e], __uint_as_float(v[4 * q + e]));
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(BNT));
+}
+
+
+
 // v1 (single-thread-group staging, kept as the reference the layout probe
 // tools/ubench/tc_dump.cu exercises; the library runs lud_tc_update2 above).
 #ifndef RG_LUD_KC
@@ -512,10 +718,10 @@ constexpr size_t smem_bytes2() { return (size_t)NS2 * 4 * BM * KC2 * 4 + 128; }
 constexpr int KC_MAIN = RG_LUD_KC;  // K chunk per stage: 16 -> 64 KB smem, 3 CTAs per SM
 constexpr size_t smem_bytes(int kc) { return (size_t)2 * 4 * BM * kc * 4 + 64; }
 
-inline Rect make_rect(int r0, int c0, int m, int nn, int k0, int kk) {
+inline Rect make_rect(int r0, int c0, int m, int nn, int k0, int kk, int bn = BN) {
     Rect r;
     r.r0 = r0; r.c0 = c0; r.m = m; r.nn = nn; r.k0 = k0; r.kk = kk;
-    r.tiles_x = (nn + BN - 1) / BN;
+    r.tiles_x = (nn + bn - 1) / bn;
     r.tiles = r.tiles_x * ((m + BM - 1) / BM);
     return r;
 }
