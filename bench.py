@@ -536,6 +536,33 @@ def run_ours(args):
             comm.hotspot(t, p, out, N, iters, coeffs=coef, g=gg, stream=stream)
     del T, P
 
+    # ---- TDO confirmation (1 GPU): the tuner times 24-step windows, which the power-capped clock
+    # makes noisy (~5-10 %); re-time its 4 best candidates on full solves, interleaved, and keep
+    # the fastest (the paper's TDO takes a median of repeated runs)
+    if ws == 1 and tune_rows:
+        ok_rows = sorted((r for r in tune_rows if r["status"] == 0 and r["median_ms"] > 0), key=lambda r: r["median_ms"])
+        cands = [rg.gran(*r["g"]) for r in ok_rows[:4]]
+        if len(cands) > 1:
+            times = {c.astuple(): [] for c in cands}
+            for c in cands:
+                step(c)  # warm (plans, graphs)
+            for _ in range(2):
+                for c in cands:
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                    step(c)
+                    e1.record(stream)
+                    torch.cuda.synchronize()
+                    times[c.astuple()].append(e0.elapsed_time(e1))
+            best_c = min(cands, key=lambda c: min(times[c.astuple()]))
+            if tuning is not None:
+                tuning["confirm"] = {"candidates": [list(c.astuple()) for c in cands],
+                                     "best_ms": [round(min(times[c.astuple()]), 3) for c in cands],
+                                     "tdo_best": list(g.astuple()), "chosen": list(best_c.astuple())}
+            g = best_c
+            step = (lambda gg=g: rg.rodinia_hotspot(t, p, iters, coeffs=coef, g=gg, out=out, scratch=scr,
+                                                    stream=stream))
+
     # ---- timed region (device events, max over ranks)
     _barrier(ws)
     torch.cuda.synchronize()
