@@ -335,7 +335,6 @@ __device__ __forceinline__ void hs_stream_body(const float* __restrict__ tin,
             for (int v = 0; v < V; ++v) ring[l][k][v] = 0.0f;
     const int ystart = y0 - H;
     const int nsteps = (y1 - y0) + 2 * H;
-#pragma unroll
     // fast-path source pointers (only dereferenced when !EC && !ER: all requested rows exist)
     const float* tsrc = tin + (size_t)max(ystart, 0) * C + col0;
     const float* psrc = pw + (size_t)max(ystart - 1, 0) * C + col0;
