@@ -142,3 +142,22 @@ def test_layout_block_cyclic():
             assert rg.dist.lud_layout(n, prow, pcol, r) == (len(_idx(n, prow, r // pcol)), len(_idx(n, pcol, r % pcol)))
     with pytest.raises(rg.RodiniaError):
         rg.dist.lud_layout(100, 2, 2, 4)
+
+
+def test_lud_dist_argument_validation_without_device():
+    # rodinia_lud_dist refuses a process grid that does not match the communicator, null local
+    # matrices and bad sizes before any CUDA call (no device needed)
+    import ctypes
+
+    import paper_conf_cgo_ivanovzdem24_b200 as rg
+    h = ctypes.c_void_p()
+    assert rg.lib.rodinia_comm_init_local(ctypes.byref(h), 4) == rg.RODINIA_OK
+    try:
+        arr = (ctypes.c_void_p * 4)(1, 1, 1, 1)
+        a = ctypes.cast(arr, ctypes.c_void_p)
+        assert rg.lib.rodinia_lud_dist(h, a, 256, 1, 3, None) == rg.RODINIA_E_INVALID  # 1 x 3 != 4
+        assert rg.lib.rodinia_lud_dist(h, a, 0, 2, 2, None) == rg.RODINIA_E_INVALID
+        assert rg.lib.rodinia_lud_dist(h, None, 256, 2, 2, None) == rg.RODINIA_E_INVALID
+        assert rg.lib.rodinia_lud_dist(None, a, 256, 2, 2, None) == rg.RODINIA_E_INVALID
+    finally:
+        rg.lib.rodinia_comm_destroy(h)
