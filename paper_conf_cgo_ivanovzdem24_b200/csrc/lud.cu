@@ -1344,6 +1344,8 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
                       int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio) {
     static bool attr = false;
     if (!attr) {
+        RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)tc::Upd3<64>::smem()));
         RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)tc::Upd3<128>::smem()));
         RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<256>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1360,7 +1362,9 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
             wide = wide && rect[i][3] > 128;
         }
     if (live == 0) return RODINIA_OK;
-    const int bn = wide ? 256 : 128;
+    // the thin next-block update (on the factorisation's critical chain): 128 x 64 tiles, twice
+    // as many CTAs of half the work
+    const int bn = wide ? 256 : 64;
     tc::Args a;
     a.nrect = 0;
     for (int i = 0; i < nr && i < 2; ++i)  // rect[i] = {r0, m, c0, nn}
@@ -1372,7 +1376,7 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
     if (wide)
         tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);
     else
-        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<128>, dim3(grid), dim3(128), tc::Upd3<128>::smem(), slot, lda, a, im);
+        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<64>, dim3(grid), dim3(128), tc::Upd3<64>::smem(), slot, lda, a, im);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;

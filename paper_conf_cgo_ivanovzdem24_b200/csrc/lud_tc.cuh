@@ -511,7 +511,7 @@ constexpr size_t smem_bytes2() { return (size_t)NS2 * 4 * BM * KC2 * 4 + 128; }
 // (3 stages at 128 columns, 2 at 256: 96 KB, 2 CTAs and 2 x BNT <= 512 TMEM columns per SM).
 template <int BNT>
 struct Upd3 {
-    static constexpr int NS = BNT == 128 ? 3 : 2;
+    static constexpr int NS = BNT == 256 ? 2 : 3;
     static constexpr int PA = BM * KC2 * 4;
     static constexpr int PB = BNT * KC2 * 4;
     static constexpr int STAGE = 2 * PA + 2 * PB;
@@ -620,14 +620,15 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
         constexpr int PITCH = 128 * 4 + 16;  // 528 B: conflict-free 16-byte row-per-lane stores
         uint8_t* row_s = sm + (warp * 32 + lane) * PITCH;
 #pragma unroll 1
-        for (int h = 0; h < BNT / 128; ++h) {
-            const int nh = min(128, ncols - 128 * h);
+        constexpr int HALF = BNT < 128 ? BNT : 128;  // columns staged per pass
+        for (int h = 0; h < BNT / HALF; ++h) {
+            const int nh = min(HALF, ncols - HALF * h);
             if (nh <= 0) break;  // CTA-uniform
             if (h > 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // row_s is free again
 #pragma unroll 1
-            for (int jb = 0; jb < 4; ++jb) {
+            for (int jb = 0; jb < HALF / 32; ++jb) {
                 uint32_t v[32];
-                const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(128 * h + jb * 32);
+                const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(HALF * h + jb * 32);
                 asm volatile(
                     "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
                     "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
@@ -655,7 +656,7 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             if (r < rend)
                 asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
-                                 A + (size_t)r * n + col0 + 128 * h),
+                                 A + (size_t)r * n + col0 + HALF * h),
                              "r"(smem_u32(row_s)), "r"(nh * 4)
                              : "memory");
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
