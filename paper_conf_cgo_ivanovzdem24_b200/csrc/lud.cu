@@ -457,6 +457,7 @@ namespace tc {
 struct Lnch {
     cudaStream_t s;
     int prio;   // cudaLaunchAttributePriority value (0 = default)
+    bool pdl = false;  // programmatic dependent of the previous kernel on the stream
 };
 template <typename... KArgs, typename... Args>
 inline void launch_p(const Lnch& L, void (*fn)(KArgs...), dim3 grid, dim3 block, size_t smem, Args... args) {
@@ -465,11 +466,20 @@ inline void launch_p(const Lnch& L, void (*fn)(KArgs...), dim3 grid, dim3 block,
     cfg.blockDim = block;
     cfg.dynamicSmemBytes = smem;
     cfg.stream = L.s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributePriority;
-    at[0].val.priority = L.prio;
+    cudaLaunchAttribute at[2];
+    int na = 0;
+    if (L.prio) {
+        at[na].id = cudaLaunchAttributePriority;
+        at[na].val.priority = L.prio;
+        ++na;
+    }
+    if (L.pdl) {
+        at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[na].val.programmaticStreamSerializationAllowed = 1;
+        ++na;
+    }
     cfg.attrs = at;
-    cfg.numAttrs = L.prio ? 1 : 0;
+    cfg.numAttrs = na;
     cudaLaunchKernelEx(&cfg, fn, (KArgs)args...);
 }
 
@@ -946,6 +956,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     float* T = S + 132 * LD;
     float* LT = T + 128 * LD;  // the current sub-panel's L columns, transposed (rows >= r stay 0)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // (a programmatic dependent on the panel-128 chain)
 #ifdef RG_LUD_PROBE
     long long pr[16] = {0}, pw[16] = {0};
 #endif
@@ -1111,6 +1122,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
         __syncthreads();
         LUD_PROBE(5 + 3 * (p / 32));
     }
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the solves may launch (they wait)
     // outputs: bulk stores of the row-major image, 1/u and the A rows first, then the transposed
     // image built in shared memory meanwhile
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -1206,6 +1218,7 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
     constexpr int LD = D128_LD;
     extern __shared__ __align__(128) float sm[];
     __shared__ __align__(8) uint64_t mbar;
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     const ldist::TrsmJob& jb = jobs.j[blockIdx.y];
     if ((int)blockIdx.x * TR_T >= jb.count) return;
     float* __restrict__ A = *jb.slot + jb.off;
@@ -1233,6 +1246,7 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
 #pragma unroll 1
     for (int p = 0; p < 128; p += 32) {
         if (p + 32 < 128) trsm_load(A, lda, lower, vec, own, idx, p + 32, xn);
+        else asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // last piece
         for (int b = 0; b < p / 32; ++b) {  // the rows of earlier blocks: columns p.. of row k
             const float* mb = M + bup_row(32 * b) + (p - 32 * b);
             const int lb = 128 - 32 * b;
@@ -1306,7 +1320,7 @@ rodinia_status diag(float* const* slot, size_t off, int lda, int r, float* mimg,
                                      (int)d128_smem()));
         attr = true;
     }
-    tc::launch_p(tc::Lnch{s, prio}, lud_diag128, dim3(1), dim3(256), d128_smem(), slot, off, lda, r, mimg);
+    tc::launch_p(tc::Lnch{s, prio, prio != 0}, lud_diag128, dim3(1), dim3(256), d128_smem(), slot, off, lda, r, mimg);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;
@@ -1328,7 +1342,7 @@ rodinia_status trsm(const TrsmJob* job, int njobs, const float* mimg, cudaStream
             cmax = std::max(cmax, job[i].count);
         }
     if (nj == 0) return RODINIA_OK;
-    tc::launch_p(tc::Lnch{s, prio}, lud_trsm128, dim3((cmax + TR_T - 1) / TR_T, nj), dim3(TR_T), trsm_smem(), js, mimg);
+    tc::launch_p(tc::Lnch{s, prio, prio != 0}, lud_trsm128, dim3((cmax + TR_T - 1) / TR_T, nj), dim3(TR_T), trsm_smem(), js, mimg);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;
@@ -1376,7 +1390,7 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
     if (wide)
         tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);
     else
-        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<64>, dim3(grid), dim3(128), tc::Upd3<64>::smem(), slot, lda, a, im);
+        tc::launch_p(tc::Lnch{s, prio, prio != 0}, tc::lud_tc_update3<64>, dim3(grid), dim3(128), tc::Upd3<64>::smem(), slot, lda, a, im);
     RG_CUDA(cudaGetLastError());
     count_launch();
     return RODINIA_OK;

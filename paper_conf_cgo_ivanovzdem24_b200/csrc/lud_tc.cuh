@@ -540,6 +540,7 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
     uint64_t* empty = full + NS;
     uint64_t* done = empty + NS;
     uint32_t* tslot = reinterpret_cast<uint32_t*>(done + 1);
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // (a programmatic dependent on the chain)
     float* A = *slot;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
@@ -609,6 +610,7 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
     __syncwarp();
     mbar_wait(done, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");  // the next kernel may launch (it waits)
 
     const int r = row0 + warp * 32 + lane;
     const int ncols = min(BNT, cend - col0);
