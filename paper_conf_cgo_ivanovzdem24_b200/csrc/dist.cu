@@ -864,7 +864,7 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
         const int bk = (int)std::min<int64_t>(NB, n - k * NB);
         const int64_t lrk = (k / prow) * NB, lck = (k / pcol) * NB;  // block (k, k) on its owner
         const int par = (int)(k & 1);
-        if (LudRank* o = find(root)) LD_TRY(ldist::diag(o->slot, (size_t)(lrk * o->nloc + lck), (int)o->nloc, bk, o->mimg, s));
+        if (LudRank* o = find(root)) LD_TRY(ldist::diag(o->slot, (size_t)(lrk * o->nloc + lck), (int)o->nloc, bk, o->mimg, s, prio_hi));
         if (k == nb - 1) break;
         // 1. the diagonal block's images to every rank
         if (P > 1) {
@@ -892,7 +892,7 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
             if (x.pr == pk && x.nloc > lc0)
                 jobs[nj++] = ldist::TrsmJob{x.slot, (size_t)(lrk * x.nloc + lc0), (int)x.nloc, 0, (int)(x.nloc - lc0), x.ib[par],
                                             ldist::img_groups(x.nloc - lc0)};
-            LD_TRY(ldist::trsm(jobs, nj, x.mimg, s));
+            LD_TRY(ldist::trsm(jobs, nj, x.mimg, s, prio_hi));
         }
         // 3. L images along process rows (from (pr, qk)), U images along process columns (from (pk, pc))
         if (P > 1) {
@@ -953,7 +953,7 @@ extern "C" rodinia_status rodinia_lud_dist(rodinia_comm* c, void* a_local, int64
                 const int ga = ldist::img_groups(rows), gb = ldist::img_groups(cols);
                 const int next[2][4] = {{(int)lr0, (int)rows, (int)lc0, (int)nbk},                 // column k+1
                                         {(int)lr0, (int)mb, (int)(lc0 + nbk), (int)(cols - nbk)}};  // row k+1
-                LD_TRY(ldist::update(x.slot, (int)x.nloc, next, 2, (int)lr0, x.ia[par], ga, (int)lc0, x.ib[par], gb, s));
+                LD_TRY(ldist::update(x.slot, (int)x.nloc, next, 2, (int)lr0, x.ia[par], ga, (int)lc0, x.ib[par], gb, s, prio_hi));
                 const int rest[1][4] = {{(int)(lr0 + mb), (int)(rows - mb), (int)(lc0 + nbk), (int)(cols - nbk)}};
                 LD_TRY(ldist::update(x.slot, (int)x.nloc, rest, 1, (int)lr0, x.ia[par], ga, (int)lc0, x.ib[par], gb, s2));
             }
