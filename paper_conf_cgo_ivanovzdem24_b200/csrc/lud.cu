@@ -956,8 +956,13 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     float* T = S + 132 * LD;
     float* LT = T + 128 * LD;  // the current sub-panel's L columns, transposed (rows >= r stay 0)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+#ifdef RG_LUD_PROBE
+    unsigned long long gt0, gt1, gt2;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt0));
+#endif
     asm volatile("griddepcontrol.wait;" ::: "memory");  // (a programmatic dependent on the panel-128 chain)
 #ifdef RG_LUD_PROBE
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt1));
     long long pr[16] = {0}, pw[16] = {0};
 #endif
     LUD_PROBE(0);
@@ -1086,35 +1091,41 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
             // rank-32 update of the rest of [nb, r)^2: units of 4 rows x 8 columns, consecutive lanes
             // on consecutive row groups of one column group (u rows broadcast, LT rows 128-bit);
             // units may reach into the zero padding (rows < 132, columns < LD): 0 - 0 * u
+            // warp 4 shares warp 0's scheduler (warp w issues on SMSP w mod 4) and stays out, so the
+            // factorisation's dependent chain keeps its issue slots; products on the FP32x2 pipe
+            // (FFMA2: element-wise the same RN fused multiply-adds, same bits)
             const int nrg = (rest + 3) / 4, ncg = (rest + 7) / 8;
-            for (int t = tid - 32; t < nrg * ncg; t += 224) {
+            const int widx = warp < 4 ? warp - 1 : warp - 2;
+            for (int t = warp == 4 ? nrg * ncg : widx * 32 + lane; t < nrg * ncg; t += 192) {
                 const int cg = t / nrg, rg = t - cg * nrg;
                 if (rg < 8 && cg < 4) continue;  // the next diagonal sub-block (warp 0)
                 const int i0 = nb + 4 * rg, j0 = nb + 8 * cg;
-                float acc[4][8];
+                float2 acc[4][4];
 #pragma unroll
                 for (int a = 0; a < 4; ++a) {
                     const float4 v0 = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0);
                     const float4 v1 = *reinterpret_cast<const float4*>(S + (i0 + a) * LD + j0 + 4);
-                    acc[a][0] = v0.x; acc[a][1] = v0.y; acc[a][2] = v0.z; acc[a][3] = v0.w;
-                    acc[a][4] = v1.x; acc[a][5] = v1.y; acc[a][6] = v1.z; acc[a][7] = v1.w;
+                    acc[a][0] = make_float2(v0.x, v0.y); acc[a][1] = make_float2(v0.z, v0.w);
+                    acc[a][2] = make_float2(v1.x, v1.y); acc[a][3] = make_float2(v1.z, v1.w);
                 }
 #pragma unroll 4
                 for (int k = 0; k < 32; ++k) {
                     const float4 u0 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
                     const float4 u1 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0 + 4);
                     const float4 l4 = *reinterpret_cast<const float4*>(LT + k * D128_LT + i0);
-                    const float u[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-                    const float l[4] = {-l4.x, -l4.y, -l4.z, -l4.w};
+                    const float2 u[4] = {make_float2(u0.x, u0.y), make_float2(u0.z, u0.w), make_float2(u1.x, u1.y),
+                                         make_float2(u1.z, u1.w)};
+                    const float2 l[4] = {make_float2(-l4.x, -l4.x), make_float2(-l4.y, -l4.y), make_float2(-l4.z, -l4.z),
+                                         make_float2(-l4.w, -l4.w)};
 #pragma unroll
                     for (int a = 0; a < 4; ++a)
 #pragma unroll
-                        for (int b = 0; b < 8; ++b) acc[a][b] = __fmaf_rn(l[a], u[b], acc[a][b]);
+                        for (int b = 0; b < 4; ++b) acc[a][b] = __ffma2_rn(l[a], u[b], acc[a][b]);
                 }
 #pragma unroll
                 for (int a = 0; a < 4; ++a) {
-                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0) = make_float4(acc[a][0], acc[a][1], acc[a][2], acc[a][3]);
-                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0 + 4) = make_float4(acc[a][4], acc[a][5], acc[a][6], acc[a][7]);
+                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0) = make_float4(acc[a][0].x, acc[a][0].y, acc[a][1].x, acc[a][1].y);
+                    *reinterpret_cast<float4*>(S + (i0 + a) * LD + j0 + 4) = make_float4(acc[a][2].x, acc[a][2].y, acc[a][3].x, acc[a][3].y);
                 }
             }
             LUD_PROBE_W(p / 32);
@@ -1162,6 +1173,9 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // shared memory read before exit
 #ifdef RG_LUD_PROBE
     LUD_PROBE(14);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt2));
+    if (tid == 0) printf("diag128 ns: wait %llu body %llu start %llu cyc %lld p0 %lld p1 %lld p2 %lld out %lld\n", gt1 - gt0, gt2 - gt1, gt0,
+                         pr[14] - pr[0], pr[5] - pr[2], pr[8] - pr[5], pr[11] - pr[8], pr[14] - pr[11]);
     if (tid == 32) printf("diag128 rest-update end (warp 1): %lld %lld %lld\n", pw[0], pw[1], pw[2]);
     __syncthreads();
     if (tid == 0)

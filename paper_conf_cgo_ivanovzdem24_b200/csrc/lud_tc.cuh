@@ -623,6 +623,11 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
         uint8_t* row_s = sm + (warp * 32 + lane) * PITCH;
 #pragma unroll 1
         constexpr int HALF = BNT < 128 ? BNT : 128;  // columns staged per pass
+        // C is read-modified-written once per update: mark it first to go from L2, so the
+        // concurrently running chain kernels keep their code and operands there (their cold
+        // instruction fetches otherwise come from HBM behind this stream)
+        uint64_t c_policy;
+        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(c_policy));
         for (int h = 0; h < BNT / HALF; ++h) {
             const int nh = min(HALF, ncols - HALF * h);
             if (nh <= 0) break;  // CTA-uniform
@@ -657,9 +662,9 @@ __global__ void __launch_bounds__(128) lud_tc_update3(float* const* __restrict__
             // generic-proxy writes -> async proxy (bulk copy engine) reads
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             if (r < rend)
-                asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
-                                 A + (size_t)r * n + col0 + HALF * h),
-                             "r"(smem_u32(row_s)), "r"(nh * 4)
+                asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.L2::cache_hint.add.f32 [%0], [%1], %2, %3;"
+                             ::"l"(A + (size_t)r * n + col0 + HALF * h),
+                             "r"(smem_u32(row_s)), "r"(nh * 4), "l"(c_policy)
                              : "memory");
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         }
