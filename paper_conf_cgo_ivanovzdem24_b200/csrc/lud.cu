@@ -997,23 +997,13 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
     if (bulk) tc::mbar_wait(&mbar, 0);
     __syncthreads();
     LUD_PROBE(1);
-    if (warp == 0) {  // the first diagonal sub-block
-        float a[32];
-#pragma unroll
-        for (int q = 0; q < 8; ++q) {
-            const float4 t = *reinterpret_cast<const float4*>(S + lane * LD + 4 * q);
-            a[4 * q] = t.x; a[4 * q + 1] = t.y; a[4 * q + 2] = t.z; a[4 * q + 3] = t.w;
-        }
-        diag32_factor(a, min(32, r), lane, rinv);
-#pragma unroll
-        for (int q = 0; q < 8; ++q)
-            *reinterpret_cast<float4*>(S + lane * LD + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
-    }
-    __syncthreads();
-    LUD_PROBE(2);
+    // p = -32 factors the first diagonal sub-block only: one inlined copy of the factorisation
+    // (the kernel's speed depends on instruction fetch)
 #pragma unroll 1
-    for (int p = 0; p + 32 < r; p += 32) {
+    for (int p = -32; p + 32 < r; p += 32) {
         const int rest = r - p - 32;  // rows below / columns right of the factored sub-block
+        const int nb = p + 32;
+        if (p >= 0) {
         if (tid < rest) {
             // L row i: x_j = (a_ij - sum_{k<j} x_k u_kj) / u_jj over the sub-block's columns
             float* xr = S + (p + 32 + tid) * LD + p;
@@ -1056,7 +1046,6 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
         }
         __syncthreads();
         LUD_PROBE(3 + 3 * (p / 32));
-        const int nb = p + 32;
         {
             // the next diagonal sub-block's rank-32 update first, by all threads (4 elements each)
             const int i = nb + (tid >> 3), j0 = nb + 4 * (tid & 7);
@@ -1073,6 +1062,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
             *reinterpret_cast<float4*>(S + i * LD + j0) = c;
         }
         __syncthreads();
+        }
         if (warp == 0) {
             // ... then its factorisation, while the other warps update the rest
             float a[32];
@@ -1081,13 +1071,13 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                 const float4 c = *reinterpret_cast<const float4*>(S + (nb + lane) * LD + nb + 4 * q);
                 a[4 * q] = c.x; a[4 * q + 1] = c.y; a[4 * q + 2] = c.z; a[4 * q + 3] = c.w;
             }
-            LUD_PROBE(4 + 3 * (p / 32));
+            if (p >= 0) LUD_PROBE(4 + 3 * (p / 32));
             diag32_factor(a, min(32, rest), lane, rinv + nb);
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(S + (nb + lane) * LD + nb + 4 * q) =
                     make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
-        } else {
+        } else if (p >= 0) {
             // rank-32 update of the rest of [nb, r)^2: units of 4 rows x 8 columns, consecutive lanes
             // on consecutive row groups of one column group (u rows broadcast, LT rows 128-bit);
             // units may reach into the zero padding (rows < 132, columns < LD): 0 - 0 * u
