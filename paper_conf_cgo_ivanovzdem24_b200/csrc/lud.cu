@@ -916,18 +916,31 @@ __device__ __forceinline__ float div_rcp(float a, float b, float rb) {
 }
 
 // Right-looking LU of the rs x rs leading part of a 32 x 32 block held one row per lane
-// (a[j] = element (lane, j)), one warp.  Step kk: row kk (final) is broadcast from lane kk
-// with warp shuffles, lanes kk < i < rs form l_ik = a_ik / u_kk and subtract l_ik u_kj for
+// (a[j] = element (lane, j)), one warp.  Step kk: row kk (final) is broadcast from lane kk,
+// lanes kk < i < rs form l_ik = a_ik / u_kk and subtract l_ik u_kj for
 // j > kk (others use l = 0: row unchanged).
 // rinv[i] = RN(1/u_ii) for i < rs.
-__device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rinv) {
+// The row is published through the block's own rows in shared memory (sb, row stride ld): lane
+// kk stores its row, the warp reads it back as 128-bit broadcasts -- a third of the code of a
+// shuffle broadcast, whose per-shuffle convergence fallback ptxas duplicates (the kernel's speed
+// depends on instruction fetch).  Lane kk's stored row is final.
+__device__ __forceinline__ void diag32_factor(float (&a)[32], int rs, int lane, float* rinv, float* sb, int ld) {
     float myrb = 0.f;
 #pragma unroll
     for (int kk = 0; kk < 32; ++kk) {
         if (kk >= rs) break;  // uniform
         float u[32];
+        if (lane == kk) {
 #pragma unroll
-        for (int j = kk; j < 32; ++j) u[j] = __shfl_sync(0xffffffffu, a[j], kk);  // row kk, broadcast
+            for (int q = kk / 4; q < 8; ++q)
+                *reinterpret_cast<float4*>(sb + kk * ld + 4 * q) = make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int q = kk / 4; q < 8; ++q) {  // row kk, broadcast
+            const float4 t = *reinterpret_cast<const float4*>(sb + kk * ld + 4 * q);
+            u[4 * q] = t.x; u[4 * q + 1] = t.y; u[4 * q + 2] = t.z; u[4 * q + 3] = t.w;
+        }
         const float rb = __frcp_rn(u[kk]);
         if (lane == kk) myrb = rb;
         const bool below = lane > kk && lane < rs;
@@ -1072,7 +1085,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                 a[4 * q] = c.x; a[4 * q + 1] = c.y; a[4 * q + 2] = c.z; a[4 * q + 3] = c.w;
             }
             if (p >= 0) LUD_PROBE(4 + 3 * (p / 32));
-            diag32_factor(a, min(32, rest), lane, rinv + nb);
+            diag32_factor(a, min(32, rest), lane, rinv + nb, S + nb * LD + nb, LD);
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(S + (nb + lane) * LD + nb + 4 * q) =
