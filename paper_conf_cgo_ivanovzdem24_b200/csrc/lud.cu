@@ -488,21 +488,72 @@ inline void launch_p(const Lnch& L, void (*fn)(KArgs...), dim3 grid, dim3 block,
 // A_kk -> lud_trsm128 solves L21 and U12 in one launch, writing the operand images (double-
 // buffered by k's parity) -> the rank-128 update of block row / column k+1 (after the previous
 // remainder); side branch: the remainder update [e2, n)^2, concurrent with the next block's
-// diag/trsm.  Returns the launch count.
-inline int launch_all3(float* const* slot, int n, float* const imgs[4], float* mimg, cudaStream_t cs, cudaStream_t cs2,
-                       cudaEvent_t ev_fork, cudaEvent_t ev_img, cudaEvent_t ev_rest, int prio_hi) {
+// diag/trsm.
+// While the trailing matrix is large (remainder update longer than the chain) the block columns
+// go in pairs (k, k+1): the main branch updates block rows/columns k+1 AND k+2 with step k's
+// panels (a 256-wide band), factors and solves k+1 into chunks 8..15 of the same pair image, and
+// updates block row/column k+2 with them; the side branch then applies both steps to
+// [e + 256, n)^2 as ONE rank-256 update -- the trailing matrix's read-modify-write (what bounds
+// that phase) once per two steps.  pairs_until: pair while n - e >= pairs_until.
+// Returns the launch count.
+inline int launch_all3(float* const* slot, int n, float* const imgs[4], float* const pimgs[4], float* mimg,
+                       cudaStream_t cs, cudaStream_t cs2, cudaEvent_t ev_fork, cudaEvent_t ev_img,
+                       cudaEvent_t ev_rest, int prio_hi, int pairs_until) {
     constexpr int NB = ldist::NB;
     int launches = 0;
     cudaEventRecord(ev_fork, cs);
     cudaStreamWaitEvent(cs2, ev_fork, 0);
     const int nb = (n + NB - 1) / NB;
     bool rest_pending = false;
+    int pair = 0;
     for (int k = 0; k < nb; ++k) {
         const int o = k * NB, bk = std::min(NB, n - o);
         ldist::diag(slot, (size_t)o * n + o, n, bk, mimg, cs, prio_hi);
         ++launches;
         if (k == nb - 1) break;
         const int e = o + NB, rows = n - e, ng = ldist::img_groups(rows);
+        if (pairs_until > 0 && rows >= pairs_until && rows > 3 * NB) {
+            // ---- steps k, k+1 as a pair (k+1 < nb - 1: rows > 2 NB)
+            float* ia = pimgs[2 * (pair & 1)];
+            float* ib = pimgs[2 * (pair & 1) + 1];
+            const size_t half = (size_t)16 * ng * tc::KC2 * 8;  // 8 chunks x hi/lo x ng groups
+            const ldist::TrsmJob jobs[2] = {{slot, (size_t)e * n + o, n, 1, rows, ia, ng},
+                                            {slot, (size_t)o * n + e, n, 0, rows, ib, ng}};
+            ldist::trsm(jobs, 2, mimg, cs, prio_hi);
+            ++launches;
+            if (rest_pending) cudaStreamWaitEvent(cs, ev_rest, 0);
+            const int e3 = e + 2 * NB;  // band: block rows / columns k+1, k+2
+            const int band[2][4] = {{e, 2 * NB, e, rows}, {e3, n - e3, e, 2 * NB}};
+            ldist::update(slot, n, band, 2, e, ia, ng, e, ib, ng, cs, prio_hi);
+            ++launches;
+            // step k+1
+            const int o1 = e, e1 = o1 + NB, rows1 = n - e1;
+            ldist::diag(slot, (size_t)o1 * n + o1, n, NB, mimg, cs, prio_hi);
+            ++launches;
+            const size_t g16 = (size_t)16 * tc::KC2 * 8;  // 128 rows = 16 groups
+            const ldist::TrsmJob jobs1[2] = {{slot, (size_t)e1 * n + o1, n, 1, rows1, ia + half + g16, ng},
+                                             {slot, (size_t)o1 * n + e1, n, 0, rows1, ib + half + g16, ng}};
+            ldist::trsm(jobs1, 2, mimg, cs, prio_hi);
+            ++launches;
+            cudaEventRecord(ev_img, cs);
+            cudaStreamWaitEvent(cs2, ev_img, 0);
+            const int e2 = e1 + NB, mb = std::min(NB, n - e1);
+            const int next[2][4] = {{e1, rows1, e1, mb}, {e1, mb, e2, n - e2}};  // block column / row k+2
+            ldist::update(slot, n, next, 2, e, ia, ng, e, ib, ng, cs, prio_hi, NB, 8);
+            ++launches;
+            if (e2 < n) {
+                const int rest[1][4] = {{e2, n - e2, e2, n - e2}};
+                ldist::update(slot, n, rest, 1, e, ia, ng, e, ib, ng, cs2, 0, 2 * NB, 0);
+                ++launches;
+                cudaEventRecord(ev_rest, cs2);
+                rest_pending = true;
+            } else {
+                rest_pending = false;
+            }
+            ++pair;
+            ++k;  // k+1 done
+            continue;
+        }
         float* ia = imgs[2 * (k & 1)];
         float* ib = imgs[2 * (k & 1) + 1];
         const ldist::TrsmJob jobs[2] = {{slot, (size_t)e * n + o, n, 1, rows, ia, ng},
@@ -681,8 +732,8 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         const void* ifn = pl.tc ? (const void*)tc::lud_tc_update2
                                 : pl.sv ? (const void*)pl.sv->fn : (const void*)pl.v->fn;
         const size_t fimg = std::max(tc::img_floats(n), ldist::img_floats(n));
-        if (pl.tc && !ge.img)  // 4 operand images + the diagonal-block payload (v3)
-            RG_CUDA(cudaMalloc(&ge.img, (4 * fimg + ldist::mimg_floats()) * sizeof(float)));
+        if (pl.tc && !ge.img)  // 4 operand images + the diagonal-block payload + 4 pair images (v3)
+            RG_CUDA(cudaMalloc(&ge.img, (12 * fimg + ldist::mimg_floats()) * sizeof(float)));
         if (!pl.tc && !ge.dscr) RG_CUDA(cudaMalloc(&ge.dscr, (size_t)m * pl.p * pl.p * sizeof(float)));
         if (pl.smem > 48 * 1024)
             RG_CUDA(cudaFuncSetAttribute(ifn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem));
@@ -702,7 +753,13 @@ rodinia_status run(float* a, int n, const Plan& pl, cudaStream_t s) {
         if (pl.tc) {
             const size_t f = fimg;
             float* const imgs[4] = {ge.img, ge.img + f, ge.img + 2 * f, ge.img + 3 * f};
-            nl = tc::launch_all3(ge.slot, n, imgs, ge.img + 4 * f, cs, cs2, ev[0], ev[1], ev[2], prio_hi);
+            float* const pb = ge.img + 4 * f + ldist::mimg_floats();
+            float* const pimgs[4] = {pb, pb + 2 * f, pb + 4 * f, pb + 6 * f};
+            // pair block columns while the trailing matrix has at least this many rows
+            const char* pe = getenv("RG_LUD_PAIR");
+            const int pairs_until = pe ? atoi(pe) : n / 2;
+            nl = tc::launch_all3(ge.slot, n, imgs, pimgs, ge.img + 4 * f, cs, cs2, ev[0], ev[1], ev[2], prio_hi,
+                                 pairs_until);
         } else {
             nl = launch_all(pl, ge.slot, n, ge.dscr, cs);
         }
@@ -1372,7 +1429,7 @@ rodinia_status set_slot(float** slot, float* a, cudaStream_t s) {
 }
 
 rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr, int a_base, const float* ia,
-                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio) {
+                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio, int kk, int c0) {
     static bool attr = false;
     if (!attr) {
         RG_CUDA(cudaFuncSetAttribute((const void*)tc::lud_tc_update3<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1400,9 +1457,9 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
     a.nrect = 0;
     for (int i = 0; i < nr && i < 2; ++i)  // rect[i] = {r0, m, c0, nn}
         if (rect[i][1] > 0 && rect[i][3] > 0)
-            a.rect[a.nrect++] = tc::make_rect(rect[i][0], rect[i][2], rect[i][1], rect[i][3], 0, LD_NB, bn);
+            a.rect[a.nrect++] = tc::make_rect(rect[i][0], rect[i][2], rect[i][1], rect[i][3], 0, kk, bn);
     if (a.nrect == 1) a.rect[1] = a.rect[0];
-    const tc::Img im{ia, ib, a_base, b_base, nga, ngb, 0};
+    const tc::Img im{ia, ib, a_base, b_base, nga, ngb, c0};
     const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
     if (wide)
         tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);

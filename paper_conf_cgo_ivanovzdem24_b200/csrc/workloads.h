@@ -92,7 +92,8 @@ rodinia_status set_slot(float** slot, float* a, cudaStream_t s);
 // A -= L U over up to two rectangles rect[i] = {r0, m, c0, nn} of the local matrix; the operand
 // images start at local row a_base / column b_base (the trailing part's first row / column)
 rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr, int a_base, const float* ia,
-                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio = 0);
+                      int nga, int b_base, const float* ib, int ngb, cudaStream_t s, int prio = 0, int kk = NB,
+                      int c0 = 0);  // kk: update rank (128, or 256 over two steps' images); c0: first image chunk
 }  // namespace ldist
 
 }  // namespace rg
