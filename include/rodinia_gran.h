@@ -220,7 +220,9 @@ rodinia_status rodinia_pathfinder_host(const int32_t* wall, int64_t rows, int64_
  * 128: per 128-wide block column the diagonal block is factored by one CTA, L21 / U12 are solved
  * one thread per row / column, and the rank-128 trailing update runs on the tensor cores
  * (tcgen05.mma kind::tf32 with the 3xTF32 split; g is ignored there); its
- * quotients are IEEE quotients formed from the pivot's correctly rounded reciprocal.
+ * quotients are IEEE quotients formed from the pivot's correctly rounded reciprocal.  While at
+ * least n/2 rows remain, two block columns share one rank-256 remainder update (environment
+ * RG_LUD_PAIR = the row threshold, 0 = off; it changes the rounding order of those updates).
  * The panel width changes fp32 rounding order and is reported separately from coarsening
  * (reading L5).  Zero pivots give inf/NaN (no pivoting, as Rodinia). */
 rodinia_status rodinia_lud(float* a, int64_t n, int32_t panel, const rodinia_granularity* g,
