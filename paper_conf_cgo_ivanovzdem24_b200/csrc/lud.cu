@@ -1462,7 +1462,7 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
     const tc::Img im{ia, ib, a_base, b_base, nga, ngb, c0};
     const int grid = a.rect[0].tiles + (a.nrect == 2 ? a.rect[1].tiles : 0);
     if (wide)
-        tc::launch_p(tc::Lnch{s, prio}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);
+        tc::launch_p(tc::Lnch{s, prio, prio != 0}, tc::lud_tc_update3<256>, dim3(grid), dim3(128), tc::Upd3<256>::smem(), slot, lda, a, im);
     else
         tc::launch_p(tc::Lnch{s, prio, prio != 0}, tc::lud_tc_update3<64>, dim3(grid), dim3(128), tc::Upd3<64>::smem(), slot, lda, a, im);
     RG_CUDA(cudaGetLastError());
