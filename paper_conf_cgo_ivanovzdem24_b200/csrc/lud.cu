@@ -1292,7 +1292,15 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
     constexpr int LD = D128_LD;
     extern __shared__ __align__(128) float sm[];
     __shared__ __align__(8) uint64_t mbar;
+#ifdef RG_LUD_PROBE
+    unsigned long long tg[8];
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tg[0]));
+#define TR_PROBE(i) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tg[i]))
+#else
+#define TR_PROBE(i)
+#endif
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    TR_PROBE(1);
     const ldist::TrsmJob& jb = jobs.j[blockIdx.y];
     if ((int)blockIdx.x * TR_T >= jb.count) return;
     float* __restrict__ A = *jb.slot + jb.off;
@@ -1316,6 +1324,7 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
     trsm_load(A, lda, lower, vec, own, idx, 0, x);
     __syncthreads();
     tc::mbar_wait(&mbar, 0);
+    TR_PROBE(2);
     float* Rt = R + tid * TR_RLD;
 #pragma unroll 1
     for (int p = 0; p < 128; p += 32) {
@@ -1377,8 +1386,18 @@ __global__ void __launch_bounds__(TR_T) lud_trsm128(TrsmJobs jobs, const float* 
         }
 #pragma unroll
         for (int q = 0; q < 16; ++q) x[q] = xn[q];
+#ifdef RG_LUD_PROBE
+        tg[3 + p / 32] = 0;
+        TR_PROBE(3 + p / 32);
+#endif
     }
+#ifdef RG_LUD_PROBE
+    if (tid == 0 && blockIdx.x == 0 && blockIdx.y == 0)
+        printf("trsm ns: count %d wait %llu mbar %llu p0 %llu p1 %llu p2 %llu p3 %llu start %llu\n", count, tg[1] - tg[0],
+               tg[2] - tg[1], tg[3] - tg[2], tg[4] - tg[3], tg[5] - tg[4], tg[6] - tg[5], tg[0]);
+#endif
 }
+#undef TR_PROBE
 
 namespace ldist {
 size_t mimg_floats() { return d128_mimg_floats(); }
