@@ -1471,6 +1471,8 @@ rodinia_status update(float* const* slot, int lda, const int (*rect)[4], int nr,
     if (live == 0) return RODINIA_OK;
     // the thin next-block update (on the factorisation's critical chain): 128 x 64 tiles, twice
     // as many CTAs of half the work
+    // (the 256-wide band of a block-column pair is on the chain too: narrow tiles there as well)
+    if (prio != 0) wide = false;
     const int bn = wide ? 256 : 64;
     tc::Args a;
     a.nrect = 0;
