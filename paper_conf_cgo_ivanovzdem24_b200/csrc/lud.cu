@@ -945,7 +945,6 @@ rodinia_status tune_lud(const rodinia_problem& pr, int reps, rodinia_granularity
 // correctly rounded reciprocal (div_rcp).
 constexpr int LD_NB = 128;
 constexpr int D128_LD = 140;                   // 16-byte rows; row-per-lane 128-bit reads conflict-free
-constexpr int D128_LT = 132;                   // transposed L sub-panel: LT[k][i]
 #ifdef RG_LUD_PROBE  // development timing probes (printf of clock64 phase stamps)
 #define LUD_PROBE(i) if (threadIdx.x == 0) pr[i] = clock64()
 #define LUD_PROBE_W(i) if (threadIdx.x == 32) pw[i] = clock64()
@@ -1020,11 +1019,12 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                                                       float* __restrict__ mimg) {
     float* A = *slot + off;  // the matrix pointer comes from a device slot (graph reuse, lud::run)
     constexpr int LD = D128_LD;
-    extern __shared__ __align__(128) float S[];  // 132 x LD, the transposed image 128 x LD, LT 32 x D128_LT
+    extern __shared__ __align__(128) float S[];  // 132 x LD, then the transposed block T 128 x LD
     __shared__ __align__(16) float rinv[128];
     __shared__ __align__(8) uint64_t mbar;
     float* T = S + 132 * LD;
-    float* LT = T + 128 * LD;  // the current sub-panel's L columns, transposed (rows >= r stay 0)
+    // T: the transposed block; the panel solves write their L columns into it as they go (row
+    // p+k of T = column p+k of L), so only the diagonal sub-blocks are transposed at the end
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 #ifdef RG_LUD_PROBE
     unsigned long long gt0, gt1, gt2;
@@ -1063,7 +1063,10 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
         if (e < 4 * LD) S[128 * LD + e] = 0.f;
         else S[((e - 4 * LD) / PADC) * LD + 128 + ((e - 4 * LD) % PADC)] = 0.f;
     }
-    for (int e = tid; e < 32 * D128_LT; e += 256) LT[e] = 0.f;
+    if (r < 128)  // columns / rows >= r of T stay zero (the update units reach into them)
+        for (int e = tid; e < 128 * LD; e += 256) T[e] = 0.f;
+    else
+        for (int e = tid; e < 128 * PADC; e += 256) T[(e / PADC) * LD + 128 + (e % PADC)] = 0.f;
     if (bulk) tc::mbar_wait(&mbar, 0);
     __syncthreads();
     LUD_PROBE(1);
@@ -1100,7 +1103,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
             for (int q = 0; q < 8; ++q)
                 *reinterpret_cast<float4*>(xr + 4 * q) = make_float4(x[4 * q], x[4 * q + 1], x[4 * q + 2], x[4 * q + 3]);
 #pragma unroll
-            for (int k = 0; k < 32; ++k) LT[k * D128_LT + p + 32 + tid] = x[k];
+            for (int k = 0; k < 32; ++k) T[(p + k) * LD + p + 32 + tid] = x[k];
         } else if (tid >= 128 && tid - 128 < rest) {
             // U column c: y_i = a_ic - sum_{k<i} l_ik y_k (unit-lower sub-block)
             const int c = p + 32 + (tid - 128);
@@ -1122,7 +1125,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
             float4 c = *reinterpret_cast<const float4*>(S + i * LD + j0);
 #pragma unroll 8
             for (int k = 0; k < 32; ++k) {
-                const float l = -LT[k * D128_LT + i];
+                const float l = -T[(p + k) * LD + i];
                 const float4 u = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
                 c.x = __fmaf_rn(l, u.x, c.x);
                 c.y = __fmaf_rn(l, u.y, c.y);
@@ -1149,7 +1152,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                     make_float4(a[4 * q], a[4 * q + 1], a[4 * q + 2], a[4 * q + 3]);
         } else if (p >= 0) {
             // rank-32 update of the rest of [nb, r)^2: units of 4 rows x 8 columns, consecutive lanes
-            // on consecutive row groups of one column group (u rows broadcast, LT rows 128-bit);
+            // on consecutive row groups of one column group (u rows broadcast, T rows 128-bit);
             // units may reach into the zero padding (rows < 132, columns < LD): 0 - 0 * u
             // warp 4 shares warp 0's scheduler (warp w issues on SMSP w mod 4) and stays out, so the
             // factorisation's dependent chain keeps its issue slots; products on the FP32x2 pipe
@@ -1172,7 +1175,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                 for (int k = 0; k < 32; ++k) {
                     const float4 u0 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0);
                     const float4 u1 = *reinterpret_cast<const float4*>(S + (p + k) * LD + j0 + 4);
-                    const float4 l4 = *reinterpret_cast<const float4*>(LT + k * D128_LT + i0);
+                    const float4 l4 = *reinterpret_cast<const float4*>(T + (p + k) * LD + i0);
                     const float2 u[4] = {make_float2(u0.x, u0.y), make_float2(u0.z, u0.w), make_float2(u1.x, u1.y),
                                          make_float2(u1.z, u1.w)};
                     const float2 l[4] = {make_float2(-l4.x, -l4.x), make_float2(-l4.y, -l4.y), make_float2(-l4.z, -l4.z),
@@ -1217,11 +1220,10 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
         }
     }
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-    for (int e = tid; e < 128 * 128; e += 256) {
-        const int i = e >> 7, k = e & 127;
+    for (int e = tid; e < 4 * 32 * 32; e += 256) {  // the diagonal sub-blocks (U and L parts)
+        const int b = e >> 10, i = 32 * b + ((e >> 5) & 31), k = 32 * b + (e & 31);
         T[k * LD + i] = S[i * LD + k];
     }
-    for (int e = tid; e < 128 * PADC; e += 256) T[(e / PADC) * LD + 128 + (e % PADC)] = 0.f;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncthreads();
     if (tid < 128) {  // packed L^T image
@@ -1245,7 +1247,7 @@ __global__ void __launch_bounds__(256, 1) lud_diag128(float* const* __restrict__
                pr[14] - pr[11], pr[3]);
 #endif
 }
-constexpr size_t d128_smem() { return ((size_t)(132 + 128) * D128_LD + 32 * D128_LT) * sizeof(float); }
+constexpr size_t d128_smem() { return (size_t)(132 + 128) * D128_LD * sizeof(float); }
 
 // Triangular solves against the factored 128 x 128 diagonal block (mimg from lud_diag128),
 // 64 threads per CTA, one thread per row (lower: L = A U^-1, row t at A + t*lda) or per
